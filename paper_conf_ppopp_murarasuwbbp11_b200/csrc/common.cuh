@@ -1,0 +1,56 @@
+// common.cuh -- shared internals of libsg (handle, errors, launch accounting).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "layout.cuh"
+
+struct sg_grid_s {
+  sg::Layout L;         // host tables
+  int device;           // device that was current at sg_create
+  sg::Layout* d_L;      // device copy of L
+};
+
+namespace sg {
+
+extern std::atomic<uint64_t> g_launches;
+inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+void set_error(const char* fmt, ...);
+sg_status cuda_fail(cudaError_t e, const char* what);
+
+// check the launch just issued; returns SG_OK or SG_ERR_CUDA
+inline sg_status launched(const char* what) {
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? SG_OK : cuda_fail(e, what);
+}
+
+constexpr int kNumSMs = 148;
+
+// ---- kernel timing instrumentation (sg_profile_enable / sg_profile_read) ----
+enum ProfKind { kProfEval = 0, kProfHier = 1 };
+struct ProfScope {  // records an event pair around the launches in its lifetime when profiling is on
+  cudaEvent_t a = nullptr, b = nullptr;
+  cudaStream_t s;
+  int kind;
+  ProfScope(int kind_, cudaStream_t s_);
+  ~ProfScope();
+};  // B200; queried at run time where it matters
+
+// ---- launchers implemented in the .cu files ---------------------------------
+sg_status launch_gp2idx(const sg_grid_s* g, const int32_t* l, const int32_t* i, uint64_t count, uint64_t* idx,
+                        cudaStream_t s);
+sg_status launch_idx2gp(const sg_grid_s* g, const uint64_t* idx, uint64_t count, int32_t* l, int32_t* i,
+                        cudaStream_t s);
+sg_status launch_coords(const sg_grid_s* g, uint64_t first, uint64_t count, void* x, sg_dtype dt, cudaStream_t s);
+sg_status launch_hierarchize(const sg_grid_s* g, void* v, sg_dtype dt, cudaStream_t s);
+size_t sfc_workspace_bytes(uint64_t m);
+sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dtype dt, void* ws, size_t ws_bytes,
+                           const uint32_t** perm_out, cudaStream_t s);
+sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
+                          void* y, sg_dtype dt, uint32_t flags, cudaStream_t s);
+
+}  // namespace sg

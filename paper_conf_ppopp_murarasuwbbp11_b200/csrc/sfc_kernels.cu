@@ -1,0 +1,97 @@
+// sfc_kernels.cu -- a1: order a query batch along a Morton (Z-order) curve.
+//
+// The paper blocks evaluation points so that a subspace brought into cache
+// serves many evaluations and copies coords coalesced to shared
+// memory.  On B200 the equivalent is spatial locality *within a
+// warp and a CTA*: queries that are close in space fall into the same cells
+// of the coarse subspaces, so their surplus gathers coalesce into few L1/L2
+// sectors.  Keys: b = min(20, 63/d) bits per dimension, interleaved with the
+// most significant bit of every dimension first; CUB radix sort of
+// (key, query index) pairs on the caller's stream.
+#include <cub/device/device_radix_sort.cuh>
+
+#include "common.cuh"
+
+namespace sg {
+
+namespace {
+
+constexpr int kThreads = 256;
+
+inline int morton_bits(int d) {
+  int b = 63 / d;
+  return b > 20 ? 20 : (b < 1 ? 1 : b);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads) k_morton(const T* __restrict__ x, uint64_t m, int d, int bits,
+                                                     uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  for (uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; q < m; q += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t c[SG_MAX_D];
+    const double scale = (double)(1u << bits);
+    const double top = scale - 1.0;
+    for (int t = 0; t < d; ++t) {
+      double v = floor((double)x[q * d + t] * scale);
+      v = v >= 0.0 ? v : 0.0;  // also maps NaN to 0
+      v = v <= top ? v : top;
+      c[t] = (uint32_t)v;
+    }
+    uint64_t key = 0;
+    for (int b = bits - 1; b >= 0; --b)
+      for (int t = 0; t < d; ++t) key = (key << 1) | ((c[t] >> b) & 1u);
+    keys[q] = key;
+    vals[q] = (uint32_t)q;
+  }
+}
+
+inline size_t align_up(size_t v) { return (v + 255) & ~(size_t)255; }
+
+size_t cub_temp_bytes(uint64_t m) {
+  size_t temp = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const uint64_t*)nullptr, (uint64_t*)nullptr,
+                                  (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)m, 0, 64);
+  return temp;
+}
+
+}  // namespace
+
+size_t sfc_workspace_bytes(uint64_t m) {
+  return 2 * align_up(m * sizeof(uint64_t)) + 2 * align_up(m * sizeof(uint32_t)) + align_up(cub_temp_bytes(m));
+}
+
+sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dtype dt, void* ws, size_t ws_bytes,
+                           const uint32_t** perm_out, cudaStream_t s) {
+  if (m > 0x7fffffffull) {
+    set_error("sg_evaluate: m = %llu exceeds 2^31-1 queries per call", (unsigned long long)m);
+    return SG_ERR_ARG;
+  }
+  if (ws_bytes < sfc_workspace_bytes(m)) {
+    set_error("sg_evaluate: workspace too small (%zu < %zu)", ws_bytes, sfc_workspace_bytes(m));
+    return SG_ERR_ARG;
+  }
+  char* p = (char*)ws;
+  uint64_t* k0 = (uint64_t*)p;
+  p += align_up(m * 8);
+  uint64_t* k1 = (uint64_t*)p;
+  p += align_up(m * 8);
+  uint32_t* v0 = (uint32_t*)p;
+  p += align_up(m * 4);
+  uint32_t* v1 = (uint32_t*)p;
+  p += align_up(m * 4);
+  size_t temp = cub_temp_bytes(m);
+  const int d = g->L.d, bits = morton_bits(d);
+  uint64_t blocks = (m + kThreads - 1) / kThreads;
+  if (blocks > (uint64_t)kNumSMs * 32) blocks = (uint64_t)kNumSMs * 32;
+  if (dt == SG_F64)
+    k_morton<double><<<(unsigned)blocks, kThreads, 0, s>>>((const double*)x, m, d, bits, k0, v0);
+  else
+    k_morton<float><<<(unsigned)blocks, kThreads, 0, s>>>((const float*)x, m, d, bits, k0, v0);
+  sg_status st = launched("k_morton");
+  if (st != SG_OK) return st;
+  cudaError_t e = cub::DeviceRadixSort::SortPairs(p, temp, k0, k1, v0, v1, (int)m, 0, d * bits, s);
+  if (e != cudaSuccess) return cuda_fail(e, "cub::DeviceRadixSort::SortPairs");
+  *perm_out = v1;
+  return SG_OK;
+}
+
+}  // namespace sg

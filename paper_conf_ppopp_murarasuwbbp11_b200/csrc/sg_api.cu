@@ -1,0 +1,381 @@
+// sg_api.cu -- the C ABI of libsg (include/sg.h): argument checking, handle
+// management, host index maps, and dispatch to the CUDA launchers.
+#include <stdarg.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "common.cuh"
+
+namespace sg {
+
+std::atomic<uint64_t> g_launches{0};
+
+static thread_local char t_err[512] = "";
+
+void set_error(const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(t_err, sizeof(t_err), fmt, ap);
+  va_end(ap);
+}
+
+// ---- profiling: event pairs recorded on the launching stream
+static std::atomic<int> g_prof_on{0};
+static std::mutex g_prof_mu;
+struct ProfRec {
+  cudaEvent_t a, b;
+  int kind;
+};
+static std::vector<ProfRec> g_prof_pending;
+static double g_prof_ms[2] = {0, 0};
+static uint64_t g_prof_n[2] = {0, 0};
+
+ProfScope::ProfScope(int kind_, cudaStream_t s_) : s(s_), kind(kind_) {
+  if (!g_prof_on.load()) return;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  cudaEventRecord(a, s);
+}
+
+ProfScope::~ProfScope() {
+  if (!a) return;
+  cudaEventRecord(b, s);
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  g_prof_pending.push_back({a, b, kind});
+}
+
+sg_status cuda_fail(cudaError_t e, const char* what) {
+  set_error("%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+  return SG_ERR_CUDA;
+}
+
+sg_status launch_eval_simple(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
+                             void* y, sg_dtype dt, cudaStream_t s);
+sg_status launch_eval_fast(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
+                           void* y, sg_dtype dt, cudaStream_t s, bool* handled);
+
+sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
+                          void* y, sg_dtype dt, uint32_t flags, cudaStream_t s) {
+  if (m == 0) return SG_OK;
+  ProfScope prof(kProfEval, s);
+  if (!(flags & SG_EVAL_GENERIC)) {
+    bool handled = false;
+    sg_status st = launch_eval_fast(g, alpha, x, perm, m, y, dt, s, &handled);
+    if (handled || st != SG_OK) return st;
+  }
+  return launch_eval_simple(g, alpha, x, perm, m, y, dt, s);
+}
+
+}  // namespace sg
+
+using namespace sg;
+
+static inline bool dtype_ok(sg_dtype dt) { return dt == SG_F64 || dt == SG_F32; }
+static inline size_t dtype_size(sg_dtype dt) { return dt == SG_F64 ? 8 : 4; }
+
+#define SG_CHECK_GRID(g)             \
+  do {                               \
+    if (!(g)) {                      \
+      set_error("NULL grid handle"); \
+      return SG_ERR_ARG;             \
+    }                                \
+  } while (0)
+
+#define SG_CHECK_DEVICE(g)                                            \
+  do {                                                                \
+    if (!(g)->d_L) {                                                  \
+      set_error("grid handle has no device (created without a GPU)"); \
+      return SG_ERR_NODEV;                                            \
+    }                                                                 \
+  } while (0)
+
+// Run device calls on the grid's device, restoring the caller's device after.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+extern "C" {
+
+sg_status sg_create(int32_t d, int32_t n, sg_grid* out, uint64_t* num_points) {
+  if (!out) {
+    set_error("sg_create: out is NULL");
+    return SG_ERR_ARG;
+  }
+  *out = nullptr;
+  if (d < 1 || d > SG_MAX_D || n < 1 || n > SG_MAX_N) {
+    set_error("sg_create: need 1 <= d <= %d and 1 <= n <= %d (got d=%d, n=%d)", SG_MAX_D, SG_MAX_N, d, n);
+    return SG_ERR_ARG;
+  }
+  sg_grid_s* g = new (std::nothrow) sg_grid_s();
+  if (!g) return SG_ERR_NOMEM;
+  if (!build_layout(d, n, &g->L)) {
+    delete g;
+    set_error("sg_create: grid d=%d n=%d has >= 2^62 points", d, n);
+    return SG_ERR_OVERFLOW;
+  }
+  g->device = -1;
+  g->d_L = nullptr;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    // host-only handle: sg_get_layout / sg_gp2idx / sg_idx2gp work, device calls return SG_ERR_NODEV
+    cudaGetLastError();
+    set_error("sg_create: no CUDA device (%s); host-only handle", e == cudaSuccess ? "count 0" : cudaGetErrorString(e));
+  } else {
+    cudaGetDevice(&g->device);
+    e = cudaMalloc((void**)&g->d_L, sizeof(Layout));
+    if (e != cudaSuccess) {
+      delete g;
+      return cuda_fail(e, "sg_create: cudaMalloc");
+    }
+    e = cudaMemcpy(g->d_L, &g->L, sizeof(Layout), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      cudaFree(g->d_L);
+      delete g;
+      return cuda_fail(e, "sg_create: cudaMemcpy");
+    }
+  }
+  *out = g;
+  if (num_points) *num_points = g->L.N;
+  return SG_OK;
+}
+
+sg_status sg_get_layout(sg_grid g, sg_layout* out) {
+  SG_CHECK_GRID(g);
+  if (!out) return SG_ERR_ARG;
+  out->d = g->L.d;
+  out->n = g->L.n;
+  out->num_points = g->L.N;
+  out->num_subspaces = g->L.T;
+  out->group_offset = g->L.off;
+  out->group_count = g->L.cnt;
+  return SG_OK;
+}
+
+sg_status sg_destroy(sg_grid g) {
+  if (!g) return SG_OK;
+  if (g->d_L) {
+    DeviceGuard guard(g->device);
+    cudaDeviceSynchronize();
+    cudaFree(g->d_L);
+  }
+  delete g;
+  return SG_OK;
+}
+
+sg_status sg_gp2idx(sg_grid g, const int32_t* l, const int32_t* i, uint64_t count, uint64_t* idx) {
+  SG_CHECK_GRID(g);
+  if (count && (!l || !i || !idx)) return SG_ERR_ARG;
+  const int d = g->L.d;
+  bool bad = false;
+  for (uint64_t q = 0; q < count; ++q) {
+    if (valid_point(g->L, l + q * d, i + q * d)) {
+      idx[q] = gp2idx(g->L, l + q * d, i + q * d);
+    } else {
+      idx[q] = UINT64_MAX;
+      bad = true;
+    }
+  }
+  if (bad) set_error("sg_gp2idx: some items are not grid points (UINT64_MAX written)");
+  return bad ? SG_ERR_RANGE : SG_OK;
+}
+
+sg_status sg_idx2gp(sg_grid g, const uint64_t* idx, uint64_t count, int32_t* l, int32_t* i) {
+  SG_CHECK_GRID(g);
+  if (count && (!l || !i || !idx)) return SG_ERR_ARG;
+  const int d = g->L.d;
+  bool bad = false;
+  for (uint64_t q = 0; q < count; ++q) {
+    if (idx[q] < g->L.N) {
+      idx2gp(g->L, idx[q], l + q * d, i + q * d);
+    } else {
+      for (int t = 0; t < d; ++t) l[q * d + t] = i[q * d + t] = -1;
+      bad = true;
+    }
+  }
+  if (bad) set_error("sg_idx2gp: some indices are >= N (-1 written)");
+  return bad ? SG_ERR_RANGE : SG_OK;
+}
+
+sg_status sg_gp2idx_device(sg_grid g, const int32_t* d_l, const int32_t* d_i, uint64_t count, uint64_t* d_idx,
+                           void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (count && (!d_l || !d_i || !d_idx)) return SG_ERR_ARG;
+  DeviceGuard guard(g->device);
+  return launch_gp2idx(g, d_l, d_i, count, d_idx, (cudaStream_t)stream);
+}
+
+sg_status sg_idx2gp_device(sg_grid g, const uint64_t* d_idx, uint64_t count, int32_t* d_l, int32_t* d_i,
+                           void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (count && (!d_l || !d_i || !d_idx)) return SG_ERR_ARG;
+  DeviceGuard guard(g->device);
+  return launch_idx2gp(g, d_idx, count, d_l, d_i, (cudaStream_t)stream);
+}
+
+sg_status sg_grid_coords_device(sg_grid g, uint64_t first, uint64_t count, void* d_x, sg_dtype dt, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (count && !d_x) return SG_ERR_ARG;
+  if (first > g->L.N || count > g->L.N - first) {
+    set_error("sg_grid_coords_device: range [%llu, +%llu) exceeds N=%llu", (unsigned long long)first,
+              (unsigned long long)count, (unsigned long long)g->L.N);
+    return SG_ERR_RANGE;
+  }
+  DeviceGuard guard(g->device);
+  return launch_coords(g, first, count, d_x, dt, (cudaStream_t)stream);
+}
+
+sg_status sg_hierarchize(sg_grid g, void* d_values, sg_dtype dt, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (!d_values) return SG_ERR_ARG;
+  DeviceGuard guard(g->device);
+  return launch_hierarchize(g, d_values, dt, (cudaStream_t)stream);
+}
+
+sg_status sg_evaluate_workspace_bytes(sg_grid g, uint64_t m, sg_dtype dt, uint32_t flags, size_t* bytes) {
+  SG_CHECK_GRID(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (!bytes) return SG_ERR_ARG;
+  *bytes = (flags & SG_EVAL_PRESORTED) || m == 0 ? 0 : sfc_workspace_bytes(m);
+  return SG_OK;
+}
+
+sg_status sg_evaluate(sg_grid g, const void* d_alpha, const void* d_x, uint64_t m, void* d_y, sg_dtype dt,
+                      uint32_t flags, void* d_workspace, size_t ws_bytes, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (m == 0) return SG_OK;
+  if (!d_alpha || !d_x || !d_y) {
+    set_error("sg_evaluate: NULL buffer");
+    return SG_ERR_ARG;
+  }
+  if (m > 0x7fffffffull) {
+    set_error("sg_evaluate: at most 2^31-1 queries per call (got %llu)", (unsigned long long)m);
+    return SG_ERR_ARG;
+  }
+  DeviceGuard guard(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const uint32_t* perm = nullptr;
+  void* own_ws = nullptr;
+  sg_status st = SG_OK;
+  if (!(flags & SG_EVAL_PRESORTED)) {
+    size_t need = sfc_workspace_bytes(m);
+    if (!d_workspace) {
+      cudaError_t e = cudaMallocAsync(&own_ws, need, s);
+      if (e != cudaSuccess) return cuda_fail(e, "sg_evaluate: cudaMallocAsync(workspace)");
+      d_workspace = own_ws;
+      ws_bytes = need;
+    }
+    st = launch_sfc_order(g, d_x, m, dt, d_workspace, ws_bytes, &perm, s);
+  }
+  if (st == SG_OK) st = launch_evaluate(g, d_alpha, d_x, perm, m, d_y, dt, flags, s);
+  if (own_ws) cudaFreeAsync(own_ws, s);
+  return st;
+}
+
+sg_status sg_evaluate_host(sg_grid g, const void* d_alpha, const void* h_x, uint64_t m, void* h_y, sg_dtype dt,
+                           uint32_t flags, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (m == 0) return SG_OK;
+  if (!d_alpha || !h_x || !h_y) return SG_ERR_ARG;
+  DeviceGuard guard(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t xb = m * (size_t)g->L.d * dtype_size(dt), yb = m * dtype_size(dt);
+  void *dx = nullptr, *dy = nullptr;
+  cudaError_t e = cudaMallocAsync(&dx, xb, s);
+  if (e != cudaSuccess) return cuda_fail(e, "sg_evaluate_host: cudaMallocAsync");
+  e = cudaMallocAsync(&dy, yb, s);
+  if (e != cudaSuccess) {
+    cudaFreeAsync(dx, s);
+    return cuda_fail(e, "sg_evaluate_host: cudaMallocAsync");
+  }
+  sg_status st = SG_OK;
+  e = cudaMemcpyAsync(dx, h_x, xb, cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) st = cuda_fail(e, "sg_evaluate_host: H2D");
+  if (st == SG_OK) st = sg_evaluate(g, d_alpha, dx, m, dy, dt, flags, nullptr, 0, stream);
+  if (st == SG_OK) {
+    e = cudaMemcpyAsync(h_y, dy, yb, cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) st = cuda_fail(e, "sg_evaluate_host: D2H");
+  }
+  cudaFreeAsync(dx, s);
+  cudaFreeAsync(dy, s);
+  e = cudaStreamSynchronize(s);
+  if (st == SG_OK && e != cudaSuccess) st = cuda_fail(e, "sg_evaluate_host: sync");
+  return st;
+}
+
+uint64_t sg_kernel_launch_count(void) { return g_launches.load(); }
+
+sg_status sg_profile_enable(int on) {
+  g_prof_on.store(on ? 1 : 0);
+  return SG_OK;
+}
+
+sg_status sg_profile_read(double* eval_ms, uint64_t* eval_launches, double* hier_ms, uint64_t* hier_launches,
+                          int reset) {
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  sg_status st = SG_OK;
+  for (auto& r : g_prof_pending) {
+    cudaError_t e = cudaEventSynchronize(r.b);
+    float ms = 0.f;
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, r.a, r.b);
+    if (e != cudaSuccess) st = cuda_fail(e, "sg_profile_read");
+    g_prof_ms[r.kind] += ms;
+    g_prof_n[r.kind] += 1;
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
+  g_prof_pending.clear();
+  if (eval_ms) *eval_ms = g_prof_ms[kProfEval];
+  if (eval_launches) *eval_launches = g_prof_n[kProfEval];
+  if (hier_ms) *hier_ms = g_prof_ms[kProfHier];
+  if (hier_launches) *hier_launches = g_prof_n[kProfHier];
+  if (reset) {
+    g_prof_ms[0] = g_prof_ms[1] = 0;
+    g_prof_n[0] = g_prof_n[1] = 0;
+  }
+  return st;
+}
+
+const char* sg_status_string(sg_status s) {
+  switch (s) {
+    case SG_OK: return "SG_OK";
+    case SG_ERR_ARG: return "SG_ERR_ARG";
+    case SG_ERR_RANGE: return "SG_ERR_RANGE";
+    case SG_ERR_OVERFLOW: return "SG_ERR_OVERFLOW";
+    case SG_ERR_NOMEM: return "SG_ERR_NOMEM";
+    case SG_ERR_CUDA: return "SG_ERR_CUDA";
+    case SG_ERR_DTYPE: return "SG_ERR_DTYPE";
+    case SG_ERR_NODEV: return "SG_ERR_NODEV";
+  }
+  return "SG_UNKNOWN";
+}
+
+const char* sg_last_error(void) { return t_err; }
+
+const char* sg_build_info(void) { return "libsg sm_100a nvcc " SG_BUILD_FLAGS; }
+
+}  // extern "C"
