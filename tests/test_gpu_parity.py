@@ -100,7 +100,7 @@ def test_device_sentinels(P, torch):
     idx = torch.tensor([0, g.num_points, -1], dtype=torch.int64, device="cuda")
     l, i = g.idx2gp(idx)
     assert (l[1:] == -1).all() and (i[1:] == -1).all() and (l[0] == 0).all()
-    lv = torch.tensor([[0, 0, 0], [3, 0, 0], [0, 0, 1]], dtype=torch.int32, device="cuda")
+    lv = torch.tensor([[0, 0, 0], [4, 0, 0], [0, 0, 1]], dtype=torch.int32, device="cuda")
     iv = torch.tensor([[1, 1, 1], [1, 1, 1], [1, 1, 4]], dtype=torch.int32, device="cuda")
     out = g.gp2idx(lv, iv)
     assert out[0].item() == 0 and out[1].item() == -1 and out[2].item() == -1
