@@ -1,0 +1,264 @@
+// eval_trie.cuh -- the evaluation hot path, v2 (rows a2-a6; Alg. 7).
+//
+// Specialised on the dimension D and a level bound NM >= n (compile time).
+// One query per thread; queries Morton-ordered (row a1).  Every lane of a
+// warp runs the SAME enumeration of level vectors in the bijection order
+// (Alg. 3: l_{D-1} slowest, l_1 fastest, l_0 implied by the group),
+// so the subspace base offset index3 + index2 is a warp-uniform running sum
+// that advances by 2^j per subspace (Alg. 7 "index2 += 2^j"); gp2idx is never
+// evaluated.  The paper's block-shared level vector becomes
+// warp-uniform control flow with no barrier.
+//
+// The level vectors of group j form a trie: dimensions D-1 .. I are runtime
+// loops (the "outer" levels), and each leaf is a *block*: every (l_{I-1}, ..,
+// l_1) with l_0 = R - l_1 - .. - l_{I-1}, R = j - sum_{t>=I} l_t, i.e.
+// C(R+I-1, I-1) subspaces that are consecutive in the layout.  A block is
+// fully unrolled for each (j, R) (compile time), so
+//   * the subspace offset of its c-th term, c * 2^j, is an immediate of the
+//     load instruction;
+//   * the in-subspace index (Alg. 5 digit order, dimension 0 most
+//     significant) costs ONE 3-input logic op per term:
+//       index1 = (C'[s] & M_row) | X_row,    s = l_1 + .. + l_{I-1},
+//     where C'[s] = ((k_0(R-s) << s) | (K_1 >> (NM-1-s))) << sigma is
+//     computed once per block for s = 0..R (it carries the digits of
+//     dimensions 0 and 1, whose levels are tied through l_0 = R - s), M_row
+//     clears the bits below (l_2 + .. + l_{I-1} + sigma), and X_row holds the
+//     digits of dimensions 2..I-1 and of the outer dimensions (P);
+//   * the address is one IMAD.WIDE (index1 * 8 + block base);
+//   * the basis product is Horner over the trie (Alg. 7's product of d hat
+//     values): acc_1 += alpha * phi_0(l_0) * phi_1(l_1) per term,
+//     one FMA per row / inner level, one per outer trie node.
+// Cells: k_t(l) = K_t >> (NM-1-l) with K_t = clamp(floor(2^{NM-1} x_t)),
+// exact.  Hat values: 2 min(u, 1-u),
+// u = 2^l x - k_t(l), exact (reading G7).  The hat values of the inner
+// dimensions live in registers, those of dimension I in shared memory
+// ([l][lane], conflict-free); dimensions > I recompute them along their
+// loop (u <- frac(2u), exact for x in [0,1), and still 0 outside).
+#pragma once
+#include "common.cuh"
+#include "eval_common.cuh"
+
+namespace sg {
+namespace trie {
+
+template <typename T, int D, int NM, int NT>
+struct Trie {
+  static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
+  static constexpr int O = D - I;          // outer (trie) dimensions
+  static constexpr int SM_PH = O > 0 ? NM : 0;      // smem rows of phi for dimension I
+  static constexpr int SM_X = O > 1 ? O - 1 : 0;    // smem rows of x for dimensions I+1..D-1
+  static constexpr size_t smem_bytes = (size_t)(SM_PH + SM_X) * NT * sizeof(T);
+
+  struct Ctx {
+    const T* __restrict__ alpha;
+    const T* phs;  // this lane's column of the dimension-I hat table
+    const T* xs;   // this lane's column of the x table of dimensions > I
+    T ph[I][NM];
+    uint32_t K[D];
+    T res;
+    uint32_t b;  // running subspace base (elements), warp-uniform
+  };
+
+  static constexpr uint32_t cnt(int R) {  // subspaces per block = C(R+I-1, I-1)
+    uint32_t c = 1;
+    for (int k = 1; k <= I - 1; ++k) c = c * (uint32_t)(R + k) / (uint32_t)k;
+    return c;
+  }
+
+  // ---------------------------------------------------------------- leaf block
+  template <int J, int R>
+  static __device__ __forceinline__ void block(Ctx& c, int sigma, uint32_t P, T prod) {
+    // per-lane block base &alpha[b + P] (P = the outer digits, all below bit
+    // sigma): per term the address is then ONE IMAD.WIDE (index1' * 8 + base)
+    // -- a warp-uniform base would force a LEA/LEA.HI.X pair per term.
+    const T* base = c.alpha + c.b + P;
+    uint32_t k0, k1, k2, k3;  // opaque copies: keep the per-block cell work inside the trie
+    asm volatile("mov.b32 %0, %1;" : "=r"(k0) : "r"(c.K[0]));
+    asm volatile("mov.b32 %0, %1;" : "=r"(k1) : "r"(c.K[I > 1 ? 1 : 0]));
+    asm volatile("mov.b32 %0, %1;" : "=r"(k2) : "r"(c.K[I > 2 ? 2 : 0]));
+    asm volatile("mov.b32 %0, %1;" : "=r"(k3) : "r"(c.K[I > 3 ? 3 : 0]));
+    const uint32_t K0R = k0 >> (NM - 1 - R);
+    uint32_t Cs[R + 1];
+#pragma unroll
+    for (int s = 0; s <= R; ++s) {
+      const uint32_t hi = K0R & ~((1u << s) - 1u);
+      const uint32_t lo = (I > 1) ? (k1 >> (NM - 1 - s)) : 0u;
+      Cs[s] = (hi | lo) << sigma;
+    }
+    constexpr int R3 = (I >= 4) ? R : 0;
+    T acc = T(0);
+    int cidx = 0;  // compile-time after unrolling: rank of the term inside the block
+#pragma unroll
+    for (int l3 = 0; l3 <= R3; ++l3) {
+      const uint32_t X3 = (I >= 4) ? ((k3 >> (NM - 1 - l3)) << sigma) : 0u;
+      const int R2 = (I >= 3) ? R - l3 : 0;
+      T acc3 = T(0);
+#pragma unroll
+      for (int l2 = 0; l2 <= R2; ++l2) {
+        const int sh = l3 + sigma;
+        uint32_t Xr = (I >= 3) ? (((k2 >> (NM - 1 - l2)) << sh) | X3) : X3;
+        asm("mov.b32 %0, %0;" : "+r"(Xr));
+        const uint32_t M = 0xffffffffu << (l2 + sh);
+        const int R1 = (I >= 2) ? R - l3 - l2 : 0;
+        T acc2 = T(0);
+#pragma unroll
+        for (int l1 = 0; l1 <= R1; ++l1) {
+          const int s = l1 + l2 + l3;
+          const int l0 = R - s;
+          uint32_t V;  // index1 = (C'[s] & M_row) | X_row: one LOP3
+          asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
+          // &alpha[b + P + index1']: one IMAD.WIDE; the term's c * 2^J is the load's immediate
+          const T* p;
+          asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
+          const T a = __ldg(p + ((uint32_t)cidx << J));
+          if (I >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[I > 1 ? 1 : 0][l1], acc2);
+          else acc2 = fma(a, c.ph[0][l0], acc2);
+          ++cidx;
+        }
+        acc3 = (I >= 3) ? fma(acc2, c.ph[I > 2 ? 2 : 0][l2], acc3) : acc2;
+      }
+      acc = (I >= 4) ? fma(acc3, c.ph[I > 3 ? 3 : 0][l3], acc) : acc3;
+    }
+    c.res = fma(acc, prod, c.res);
+    c.b += cnt(R) << J;
+  }
+
+#define SG_TRIE_CASE(r) \
+  case r:               \
+    if constexpr (r <= J) block<J, r>(c, sigma, P, prod); \
+    break;
+
+  template <int J>
+  static __device__ __forceinline__ void leaf(Ctx& c, int R, int sigma, uint32_t P, T prod) {
+    switch (R) {
+      SG_TRIE_CASE(0) SG_TRIE_CASE(1) SG_TRIE_CASE(2) SG_TRIE_CASE(3)
+      SG_TRIE_CASE(4) SG_TRIE_CASE(5) SG_TRIE_CASE(6) SG_TRIE_CASE(7)
+      SG_TRIE_CASE(8) SG_TRIE_CASE(9) SG_TRIE_CASE(10) SG_TRIE_CASE(11)
+      SG_TRIE_CASE(12) SG_TRIE_CASE(13) SG_TRIE_CASE(14) SG_TRIE_CASE(15)
+      default: break;
+    }
+  }
+#undef SG_TRIE_CASE
+
+  // ------------------------------------------------------- outer trie levels
+  // Dimension t (D-1 .. I), ascending l_t (Alg. 3 order); `budget` is what is
+  // left for dimensions t..0, sigma = sum_{u>t} l_u (the shift of dimension
+  // t's digit), P = the digits of dimensions > t, prod = their hat product.
+  template <int J, int t>
+  static __device__ __forceinline__ void outer(Ctx& c, int budget, int sigma, uint32_t P, T prod) {
+    if constexpr (O == 0) {
+      block<J, J>(c, 0, 0u, T(1));  // no outer dimensions: one block per group
+    } else if constexpr (t < I) {
+      leaf<J>(c, budget, sigma, P, prod);
+    } else if constexpr (t == I) {
+      for (int lt = 0; lt <= budget; ++lt) {
+        const T ph = c.phs[lt * NT];
+        const uint32_t kt = c.K[t] >> (NM - 1 - lt);
+        outer<J, t - 1>(c, budget - lt, sigma + lt, P | (kt << sigma), prod * ph);
+      }
+    } else {
+      T u = c.xs[(t - I - 1) * NT];  // u_l = 2^l x - k_t(l), starting at l = 0
+      for (int lt = 0; lt <= budget; ++lt) {
+        const T w = T(1) - u;
+        const T mn = u < w ? u : w;
+        T ph = mn + mn;
+        ph = ph > T(0) ? ph : T(0);
+        const uint32_t kt = c.K[t] >> (NM - 1 - lt);
+        outer<J, t - 1>(c, budget - lt, sigma + lt, P | (kt << sigma), prod * ph);
+        u = u + u;
+        u = u >= T(1) ? u - T(1) : u;
+      }
+    }
+  }
+
+  template <int J, int J1>
+  static __device__ __forceinline__ void groups(Ctx& c, int n) {
+    if constexpr (J <= J1 && J < NM) {
+      if (J < n) {
+        outer<J, D - 1>(c, J, 0, 0u, T(1));
+        groups<J + 1, J1>(c, n);
+      }
+    }
+  }
+};
+
+
+// One launch evaluates the level groups J0..J1 (compile time) for every
+// query; launches of consecutive ranges accumulate into y (accumulate = 0 for
+// the first range).  b0 = index3(J0), the offset of group J0.
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1>
+__global__ void __launch_bounds__(NT, MINB)
+    k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
+                int n, uint32_t b0, int accumulate, T* __restrict__ y) {
+  using TR = Trie<T, D, NM, NT>;
+  constexpr int I = TR::I;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* sm = reinterpret_cast<T*>(smem_raw);
+  const int tid = threadIdx.x;
+  const uint32_t q = blockIdx.x * NT + tid;
+  const bool active = q < m;
+  const uint32_t src = active ? (perm ? perm[q] : q) : 0u;
+
+  typename TR::Ctx c;
+  c.alpha = alpha;
+  c.phs = sm + tid;
+  c.xs = sm + TR::SM_PH * NT + tid;
+  // ---- a2: finest cells of every dimension; hat values of the inner ones
+  bool bad = false;
+  const T fine = (T)(1u << (NM - 1));
+#pragma unroll
+  for (int t = 0; t < D; ++t) {
+    const T xt = active ? x[(size_t)src * D + t] : T(0.5);
+    bad |= isnan(xt);
+    T kf = floor(xt * fine);
+    kf = kf > T(0) ? kf : T(0);
+    kf = kf < fine - T(1) ? kf : fine - T(1);
+    c.K[t] = (uint32_t)kf;
+    if (t < I) {
+#pragma unroll
+      for (int l = 0; l < NM; ++l) {
+        uint32_t cell;
+        c.ph[t < I ? t : 0][l] = hat_cell<T>(xt, l, cell);
+      }
+    } else if (t == I) {
+#pragma unroll
+      for (int l = 0; l < NM; ++l) {
+        uint32_t cell;
+        sm[l * NT + tid] = hat_cell<T>(xt, l, cell);
+      }
+    } else {
+      sm[(TR::SM_PH + (t - I - 1)) * NT + tid] = xt;
+    }
+  }
+  // (no barrier: every lane reads only its own shared-memory column)
+  c.res = T(0);
+  c.b = b0;
+  TR::template groups<J0, J1>(c, n);
+  if (active) {
+    T r = c.res;
+    if (accumulate) r += y[src];
+    y[src] = bad ? T(NAN) : r;
+  }
+}
+
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1>
+sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
+                       cudaStream_t s) {
+  if (J0 >= L.n) return SG_OK;
+  using TR = Trie<T, D, NM, NT>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1>;
+  const size_t smem = TR::smem_bytes;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)(smem > 48 * 1024 ? smem : 48 * 1024));
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_eval_trie)");
+    attr_set = true;
+  }
+  const unsigned blocks = (unsigned)((m + NT - 1) / NT);
+  kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, L.n, (uint32_t)L.off[J0], J0 > 0 ? 1 : 0, y);
+  return launched("k_eval_trie");
+}
+
+}  // namespace trie
+}  // namespace sg

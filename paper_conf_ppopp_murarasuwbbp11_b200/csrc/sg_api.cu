@@ -58,6 +58,8 @@ sg_status launch_eval_simple(const sg_grid_s* g, const void* alpha, const void* 
                              void* y, sg_dtype dt, cudaStream_t s);
 sg_status launch_eval_fast(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                            void* y, sg_dtype dt, cudaStream_t s, bool* handled);
+sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
+                           void* y, sg_dtype dt, cudaStream_t s, bool* handled);
 
 sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                           void* y, sg_dtype dt, uint32_t flags, cudaStream_t s) {
@@ -65,7 +67,9 @@ sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, 
   ProfScope prof(kProfEval, s);
   if (!(flags & SG_EVAL_GENERIC)) {
     bool handled = false;
-    sg_status st = launch_eval_fast(g, alpha, x, perm, m, y, dt, s, &handled);
+    sg_status st = launch_eval_trie(g, alpha, x, perm, m, y, dt, s, &handled);
+    if (handled || st != SG_OK) return st;
+    st = launch_eval_fast(g, alpha, x, perm, m, y, dt, s, &handled);
     if (handled || st != SG_OK) return st;
   }
   return launch_eval_simple(g, alpha, x, perm, m, y, dt, s);
