@@ -1,6 +1,8 @@
 // eval_trie.cu -- dispatch of the v2 evaluation kernel (eval_trie.cuh) by
 // (d, n, dtype); shapes without an instantiation return handled = false and
 // fall through to eval_fast.cu / eval_simple.cu.
+#include <stdlib.h>
+
 #include "common.cuh"
 
 namespace sg {
@@ -9,6 +11,8 @@ namespace sg {
   sg_status name(const Layout& L, const T* a, const T* x, const uint32_t* p, uint64_t m, T* y, cudaStream_t s);
 SG_DECL(trie_d10n11_a, double)
 SG_DECL(trie_d10n11_b, double)
+SG_DECL(trie_d10n11_a_mb2, double)
+SG_DECL(trie_d10n11_b_mb2, double)
 SG_DECL(trie_d2n3, double)
 SG_DECL(trie_d5n8, double)
 SG_DECL(trie_d5n10, double)
@@ -28,6 +32,11 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     const double* xx = (const double*)x;
     double* yy = (double*)y;
     if (d == 10 && n == 11) {
+      static const bool mb2 = getenv("SG_TRIE_MINB") && atoi(getenv("SG_TRIE_MINB")) == 2;  // experiment switch
+      if (mb2) {
+        sg_status st = trie_d10n11_a_mb2(L, a, xx, perm, m, yy, s);
+        return st == SG_OK ? trie_d10n11_b_mb2(L, a, xx, perm, m, yy, s) : st;
+      }
       sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
       return st == SG_OK ? trie_d10n11_b(L, a, xx, perm, m, yy, s) : st;
     }

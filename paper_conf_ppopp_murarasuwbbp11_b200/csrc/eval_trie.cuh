@@ -45,15 +45,18 @@ template <typename T, int D, int NM, int NT>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
-  static constexpr int SM_PH = O > 0 ? NM : 0;      // smem rows of phi for dimension I
-  static constexpr int SM_X = O > 1 ? O - 1 : 0;    // smem rows of x for dimensions I+1..D-1
-  static constexpr size_t smem_bytes = (size_t)(SM_PH + SM_X) * NT * sizeof(T);
+  // shared memory, [row][lane]: hat values of dimensions 2, 3 (loaded per
+  // block), of dimension I (per outer node), then x of dimensions I+1..D-1
+  static constexpr int SM_IN = 2 * NM;
+  static constexpr int SM_PH = O > 0 ? NM : 0;
+  static constexpr int SM_X = O > 1 ? O - 1 : 0;
+  static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X) * NT * sizeof(T);
 
   struct Ctx {
     const T* __restrict__ alpha;
-    const T* phs;  // this lane's column of the dimension-I hat table
+    const T* phs;  // this lane's column of the hat tables (dims 2, 3, I)
     const T* xs;   // this lane's column of the x table of dimensions > I
-    T ph[I][NM];
+    T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
     uint32_t K[D];
     T res;
     uint32_t b;  // running subspace base (elements), warp-uniform
@@ -66,58 +69,67 @@ struct Trie {
   }
 
   // ---------------------------------------------------------------- leaf block
+  // Group J, R = J - sigma: every shift below is a compile-time constant.
   template <int J, int R>
-  static __device__ __forceinline__ void block(Ctx& c, int sigma, uint32_t P, T prod) {
-    // per-lane block base &alpha[b + P] (P = the outer digits, all below bit
-    // sigma): per term the address is then ONE IMAD.WIDE (index1' * 8 + base)
-    // -- a warp-uniform base would force a LEA/LEA.HI.X pair per term.
+  static __device__ __forceinline__ void block(Ctx& c, uint32_t P, T prod) {
+    constexpr int SG = J - R;  // sigma = sum of the outer levels
+    // per-lane block base &alpha[b + P] (P = the outer digits, all below bit SG)
     const T* base = c.alpha + c.b + P;
     uint32_t k0, k1, k2, k3;  // opaque copies: keep the per-block cell work inside the trie
     asm volatile("mov.b32 %0, %1;" : "=r"(k0) : "r"(c.K[0]));
     asm volatile("mov.b32 %0, %1;" : "=r"(k1) : "r"(c.K[I > 1 ? 1 : 0]));
     asm volatile("mov.b32 %0, %1;" : "=r"(k2) : "r"(c.K[I > 2 ? 2 : 0]));
     asm volatile("mov.b32 %0, %1;" : "=r"(k3) : "r"(c.K[I > 3 ? 3 : 0]));
-    const uint32_t K0R = k0 >> (NM - 1 - R);
+    // C'[s] = (k_0(R-s) << (s+SG)) | (k_1 digits at level s, shifted by SG);
+    // bits below SG are garbage and cleared by every row mask.
+    const uint32_t K0J = k0 >> (NM - 1 - J);
     uint32_t Cs[R + 1];
 #pragma unroll
     for (int s = 0; s <= R; ++s) {
-      const uint32_t hi = K0R & ~((1u << s) - 1u);
-      const uint32_t lo = (I > 1) ? (k1 >> (NM - 1 - s)) : 0u;
-      Cs[s] = (hi | lo) << sigma;
+      const uint32_t hi = K0J & ~((1u << (s + SG)) - 1u);
+      const uint32_t lo = (I > 1) ? (k1 >> (NM - 1 - s - SG)) : 0u;
+      Cs[s] = hi | lo;
+    }
+    // hat values of dimensions 2, 3 for levels 0..R, from shared memory
+    T ph2[R + 1], ph3[R + 1];
+#pragma unroll
+    for (int l = 0; l <= R; ++l) {
+      ph2[l] = (I >= 3) ? c.phs[(0 * NM + l) * NT] : T(1);
+      ph3[l] = (I >= 4) ? c.phs[(1 * NM + l) * NT] : T(1);
     }
     constexpr int R3 = (I >= 4) ? R : 0;
     T acc = T(0);
     int cidx = 0;  // compile-time after unrolling: rank of the term inside the block
 #pragma unroll
     for (int l3 = 0; l3 <= R3; ++l3) {
-      const uint32_t X3 = (I >= 4) ? ((k3 >> (NM - 1 - l3)) << sigma) : 0u;
+      // k_3(l3) << SG
+      const uint32_t X3 = (I >= 4) ? ((k3 >> (NM - 1 - l3 - SG)) & ~((1u << SG) - 1u)) : 0u;
       const int R2 = (I >= 3) ? R - l3 : 0;
       T acc3 = T(0);
 #pragma unroll
       for (int l2 = 0; l2 <= R2; ++l2) {
-        const int sh = l3 + sigma;
-        uint32_t Xr = (I >= 3) ? (((k2 >> (NM - 1 - l2)) << sh) | X3) : X3;
+        // X_row = (k_2(l2) << (l3+SG)) | X3
+        uint32_t Xr = (I >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG)) & ~((1u << (l3 + SG)) - 1u)) | X3) : X3;
         asm("mov.b32 %0, %0;" : "+r"(Xr));
-        const uint32_t M = 0xffffffffu << (l2 + sh);
+        const uint32_t M = 0xffffffffu << (l2 + l3 + SG);
         const int R1 = (I >= 2) ? R - l3 - l2 : 0;
         T acc2 = T(0);
 #pragma unroll
         for (int l1 = 0; l1 <= R1; ++l1) {
           const int s = l1 + l2 + l3;
           const int l0 = R - s;
-          uint32_t V;  // index1 = (C'[s] & M_row) | X_row: one LOP3
+          uint32_t V;  // index1 - P = (C'[s] & M_row) | X_row: one LOP3
           asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
-          // &alpha[b + P + index1']: one IMAD.WIDE; the term's c * 2^J is the load's immediate
-          const T* p;
+          const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
           asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
           const T a = __ldg(p + ((uint32_t)cidx << J));
           if (I >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[I > 1 ? 1 : 0][l1], acc2);
           else acc2 = fma(a, c.ph[0][l0], acc2);
           ++cidx;
         }
-        acc3 = (I >= 3) ? fma(acc2, c.ph[I > 2 ? 2 : 0][l2], acc3) : acc2;
+        acc3 = (I >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
       }
-      acc = (I >= 4) ? fma(acc3, c.ph[I > 3 ? 3 : 0][l3], acc) : acc3;
+      acc = (I >= 4) ? fma(acc3, ph3[l3], acc) : acc3;
     }
     c.res = fma(acc, prod, c.res);
     c.b += cnt(R) << J;
@@ -125,7 +137,7 @@ struct Trie {
 
 #define SG_TRIE_CASE(r) \
   case r:               \
-    if constexpr (r <= J) block<J, r>(c, sigma, P, prod); \
+    if constexpr (r <= J) block<J, r>(c, P, prod); \
     break;
 
   template <int J>
@@ -147,12 +159,12 @@ struct Trie {
   template <int J, int t>
   static __device__ __forceinline__ void outer(Ctx& c, int budget, int sigma, uint32_t P, T prod) {
     if constexpr (O == 0) {
-      block<J, J>(c, 0, 0u, T(1));  // no outer dimensions: one block per group
+      block<J, J>(c, 0u, T(1));  // no outer dimensions: one block per group
     } else if constexpr (t < I) {
       leaf<J>(c, budget, sigma, P, prod);
     } else if constexpr (t == I) {
       for (int lt = 0; lt <= budget; ++lt) {
-        const T ph = c.phs[lt * NT];
+        const T ph = c.phs[(SM_IN + lt) * NT];
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
         outer<J, t - 1>(c, budget - lt, sigma + lt, P | (kt << sigma), prod * ph);
       }
@@ -202,8 +214,9 @@ __global__ void __launch_bounds__(NT, MINB)
   typename TR::Ctx c;
   c.alpha = alpha;
   c.phs = sm + tid;
-  c.xs = sm + TR::SM_PH * NT + tid;
-  // ---- a2: finest cells of every dimension; hat values of the inner ones
+  c.xs = sm + (TR::SM_IN + TR::SM_PH) * NT + tid;
+  // ---- a2: finest cells of every dimension; hat values of every level of
+  // dimensions 0..I (registers for 0, 1; shared memory for 2, 3, I)
   bool bad = false;
   const T fine = (T)(1u << (NM - 1));
 #pragma unroll
@@ -214,20 +227,17 @@ __global__ void __launch_bounds__(NT, MINB)
     kf = kf > T(0) ? kf : T(0);
     kf = kf < fine - T(1) ? kf : fine - T(1);
     c.K[t] = (uint32_t)kf;
-    if (t < I) {
+    if (t <= I) {
 #pragma unroll
       for (int l = 0; l < NM; ++l) {
         uint32_t cell;
-        c.ph[t < I ? t : 0][l] = hat_cell<T>(xt, l, cell);
-      }
-    } else if (t == I) {
-#pragma unroll
-      for (int l = 0; l < NM; ++l) {
-        uint32_t cell;
-        sm[l * NT + tid] = hat_cell<T>(xt, l, cell);
+        const T h = hat_cell<T>(xt, l, cell);
+        if (t < 2) c.ph[t < 2 ? t : 0][l] = h;
+        else if (t < I) sm[((t - 2) * NM + l) * NT + tid] = h;
+        else sm[(TR::SM_IN + l) * NT + tid] = h;
       }
     } else {
-      sm[(TR::SM_PH + (t - I - 1)) * NT + tid] = xt;
+      sm[(TR::SM_IN + TR::SM_PH + (t - I - 1)) * NT + tid] = xt;
     }
   }
   // (no barrier: every lane reads only its own shared-memory column)
@@ -253,6 +263,11 @@ sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)(smem > 48 * 1024 ? smem : 48 * 1024));
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_eval_trie)");
+    // shared memory only for the per-lane tables: the rest of the 256 KB stays L1
+    // for the surplus gathers
+    const int pct = (int)((smem * MINB * 100 + 227 * 1024 - 1) / (227 * 1024)) + 1;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, pct > 100 ? 100 : pct);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(carveout)");
     attr_set = true;
   }
   const unsigned blocks = (unsigned)((m + NT - 1) / NT);
