@@ -59,7 +59,7 @@ def peaks():
 
 def workload_config(m_per_gpu, n_gpus):
     return {"workload": "cfg3: d=10, n=11 sparse grid (127,574,017 fp64 surpluses, function A hierarchized "
-                        "each step), 1e7 uniform random queries per GPU (SplitMix64 seed 0x5EED0003+rank), "
+                        "each step), 1e7 uniform random queries per GPU (rows [rank*1e7, (rank+1)*1e7) of the SplitMix64 stream, seed 0x5EED0003), "
                         "Morton-ordered inside sg_evaluate",
             "d": CFG["d"], "n": CFG["n"], "num_points": 127574017, "queries_per_gpu": m_per_gpu,
             "global_batch": m_per_gpu * n_gpus, "parallelism": f"query-partitioned x{n_gpus}, alpha broadcast",
@@ -166,6 +166,7 @@ def run_sg(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
     import paper_conf_ppopp_murarasuwbbp11_b200 as P
+    from paper_conf_ppopp_murarasuwbbp11_b200 import multi
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
@@ -181,7 +182,8 @@ def run_sg(args, rank, world, local_rank):
         b = min(N, a + chunk)
         values[a:b] = S.f_A_torch(g.coords(a, b - a, device=dev))
     alpha = torch.empty_like(values)
-    x = S.queries_torch(d, m, CFG["seed"] + rank, device=dev)
+    first, _ = multi.shard_range(m, rank)  # rank's rows of the one global query stream
+    x = S.queries_torch(d, m, CFG["seed"], device=dev, first=first)
     y = torch.empty(m, dtype=torch.float64, device=dev)
     ws = torch.empty(g.workspace_bytes(m), dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
@@ -191,7 +193,7 @@ def run_sg(args, rank, world, local_rank):
             alpha.copy_(values)
             g.hierarchize_(alpha)
         if world > 1:
-            dist.broadcast(alpha, src=0)
+            multi.replicate_surpluses(alpha, src=0)  # the path's one collective
         g.evaluate(alpha, x, out=y, workspace=ws)
 
     def barrier():
@@ -242,7 +244,7 @@ def run_sg(args, rank, world, local_rank):
                 alpha.copy_(values_h, non_blocking=True)
                 g.hierarchize_(alpha)
             if world > 1:
-                dist.broadcast(alpha, src=0)
+                multi.replicate_surpluses(alpha, src=0)
             g.evaluate_host(alpha, x_h, y_h)  # H2D x, evaluate, D2H y, synchronizes
 
         step_e2e()

@@ -14,7 +14,7 @@ timeout 900 python bench.py --steps 3 --warmup 3 > gpurun_out/${TAG}_bench.log 2
 echo "bench exit $?" >> gpurun_out/${TAG}_bench.log
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
   python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu > gpurun_out/${TAG}_launches.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_eval -c 1 -o gpurun_out/${TAG}_eval \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_eval_trie --launch-skip 4 -c 1 -o gpurun_out/${TAG}_eval \
   python bench.py --steps 1 --warmup 0 --m $MP --no-e2e --no-cpu > gpurun_out/${TAG}_ncu_eval.log 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_hier -c 2 -o gpurun_out/${TAG}_hier \
   python bench.py --steps 1 --warmup 0 --m 100000 --no-e2e --no-cpu > gpurun_out/${TAG}_ncu_hier.log 2>&1
