@@ -2,7 +2,6 @@
 // (d, n, dtype); shapes without an instantiation return handled = false and
 // fall through to eval_fast.cu / eval_simple.cu.
 #include <stdlib.h>
-#include <string.h>
 
 #include "common.cuh"
 
@@ -12,12 +11,6 @@ namespace sg {
   sg_status name(const Layout& L, const T* a, const T* x, const uint32_t* p, uint64_t m, T* y, cudaStream_t s);
 SG_DECL(trie_d10n11_a, double)
 SG_DECL(trie_d10n11_b, double)
-SG_DECL(trie_d10n11_a_384x1, double)
-SG_DECL(trie_d10n11_b_384x1, double)
-SG_DECL(trie_d10n11_a_256x1, double)
-SG_DECL(trie_d10n11_b_256x1, double)
-SG_DECL(trie_d10n11_a_256x2, double)
-SG_DECL(trie_d10n11_b_256x2, double)
 SG_DECL(trie_d2n3, double)
 SG_DECL(trie_d5n8, double)
 SG_DECL(trie_d5n10, double)
@@ -37,19 +30,6 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     const double* xx = (const double*)x;
     double* yy = (double*)y;
     if (d == 10 && n == 11) {
-      // experiment switch: CTA shape (threads x resident CTAs per SM)
-      static const char* shape = getenv("SG_TRIE_SHAPE");
-      if (shape) {
-        sg_status (*fa)(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t) = nullptr;
-        sg_status (*fb)(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t) = nullptr;
-        if (!strcmp(shape, "384x1")) { fa = trie_d10n11_a_384x1; fb = trie_d10n11_b_384x1; }
-        if (!strcmp(shape, "256x1")) { fa = trie_d10n11_a_256x1; fb = trie_d10n11_b_256x1; }
-        if (!strcmp(shape, "256x2")) { fa = trie_d10n11_a_256x2; fb = trie_d10n11_b_256x2; }
-        if (fa) {
-          sg_status st = fa(L, a, xx, perm, m, yy, s);
-          return st == SG_OK ? fb(L, a, xx, perm, m, yy, s) : st;
-        }
-      }
       sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
       return st == SG_OK ? trie_d10n11_b(L, a, xx, perm, m, yy, s) : st;
     }

@@ -135,13 +135,111 @@ struct Trie {
     c.b += cnt(R) << J;
   }
 
+  // ------------------------------------------------------- outer trie levels
+  // node<J, t, B>: the sub-trie of dimensions t .. 0 whose levels sum to B
+  // (l_0 implied), under the outer digits P (dimensions > t, all below bit
+  // J - B) and their hat product `prod`.  B is a compile-time constant at
+  // every node, so every digit shift (J - B for dimension t) is an immediate.
+  // Small sub-tries (C(B+t, t) <= kFlat terms) are emitted as straight-line
+  // code: one basic block, all its surplus loads in flight together (the
+  // v2 trie issued them one small block at a time and was latency-bound,
+  // profiles/r01_v2_*).  Large ones loop over l_t at run time and dispatch the
+  // child's budget B - l_t through a switch.
+  static constexpr int kFlat = 70;   // straight-line sub-trie size (terms)
+  static constexpr int kFull = 4;    // dimension I: unroll every l_I when B <= kFull
+  static constexpr int kTail = 2;    // dimension I: merge the blocks R <= kTail into one basic block
+
+  static constexpr uint32_t binom(int a, int b) {
+    uint32_t c = 1;
+    for (int k = 1; k <= b; ++k) c = c * (uint32_t)(a - b + k) / (uint32_t)k;
+    return c;
+  }
+
+  // hat value from u = 2^l x - k(l) (reading G7): max(0, 2 min(u, 1-u))
+  static __device__ __forceinline__ T hat_u(T u) {
+    const T w = T(1) - u;
+    const T mn = u < w ? u : w;
+    const T h = mn + mn;
+    return h > T(0) ? h : T(0);
+  }
+  // u_{l+1} = frac(2 u_l), exact for u in [0, 1); stays outside [0,1) otherwise
+  static __device__ __forceinline__ T dbl_u(T u) {
+    u = u + u;
+    return u >= T(1) ? u - T(1) : u;
+  }
+
+  // dimension I (the innermost outer dimension) at compile-time budget B:
+  // levels l = L .. B unrolled into one basic block
+  template <int J, int B, int L>
+  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod) {
+    if constexpr (L <= B) {
+      constexpr int SG = J - B;
+      const T ph = c.phs[(SM_IN + L) * NT];
+      const uint32_t kt = c.K[I] >> (NM - 1 - L);
+      block<J, B - L>(c, P | (kt << SG), prod * ph);
+      inner_unrolled<J, B, L + 1>(c, P, prod);
+    }
+  }
+
+  // sub-trie of dimensions t .. 0 at compile-time budget B, straight-line
+  template <int J, int t, int B, int L>
+  static __device__ __forceinline__ void flat_level(Ctx& c, uint32_t P, T prod, T u) {
+    if constexpr (L <= B) {
+      constexpr int SG = J - B;
+      const uint32_t kt = c.K[t] >> (NM - 1 - L);
+      flat<J, t - 1, B - L>(c, P | (kt << SG), prod * hat_u(u));
+      if constexpr (L < B) flat_level<J, t, B, L + 1>(c, P, prod, dbl_u(u));
+    }
+  }
+  template <int J, int t, int B>
+  static __device__ __forceinline__ void flat(Ctx& c, uint32_t P, T prod) {
+    if constexpr (t < I) block<J, B>(c, P, prod);
+    else if constexpr (t == I) inner_unrolled<J, B, 0>(c, P, prod);
+    else flat_level<J, t, B, 0>(c, P, prod, c.xs[(t - I - 1) * NT]);
+  }
+  template <int t>
+  static constexpr int flat_max() {  // largest budget whose sub-trie at t is straight-line
+    if (t == I) return kFull;
+    int b = 0;
+    while (binom(b + 1 + t, t) <= (uint32_t)kFlat) ++b;
+    return b;
+  }
+
+#define SG_TRIE_FLAT(k) \
+  case k:               \
+    if constexpr (k <= FM && k <= J) flat<J, t, (k <= FM && k <= J ? k : 0)>(c, P, prod); \
+    break;
+  // dispatch a small run-time budget into the compile-time straight-line sub-tries
+  template <int J, int t>
+  static __device__ __forceinline__ void flat_dispatch(Ctx& c, int B, uint32_t P, T prod) {
+    constexpr int FM = flat_max<t>();
+    switch (B) {
+      SG_TRIE_FLAT(0) SG_TRIE_FLAT(1) SG_TRIE_FLAT(2) SG_TRIE_FLAT(3)
+      SG_TRIE_FLAT(4) SG_TRIE_FLAT(5) SG_TRIE_FLAT(6) SG_TRIE_FLAT(7)
+      default: break;
+    }
+  }
+#undef SG_TRIE_FLAT
+
+  // tail of dimension I at run-time budget B: the blocks R = RT .. 0
+  // (l_I = B - R), merged into one basic block
+  template <int J, int RT>
+  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod) {
+    if constexpr (RT >= 0) {
+      const int lt = B - RT;
+      const T ph = c.phs[(SM_IN + lt) * NT];
+      const uint32_t kt = c.K[I] >> (NM - 1 - lt);
+      block<J, RT>(c, P | (kt << (J - B)), prod * ph);
+      inner_tail<J, RT - 1>(c, B, P, prod);
+    }
+  }
+
 #define SG_TRIE_CASE(r) \
   case r:               \
-    if constexpr (r <= J) block<J, r>(c, P, prod); \
+    if constexpr (r <= J) block<J, (r <= J ? r : 0)>(c, P, prod); \
     break;
-
   template <int J>
-  static __device__ __forceinline__ void leaf(Ctx& c, int R, int sigma, uint32_t P, T prod) {
+  static __device__ __forceinline__ void leaf(Ctx& c, int R, uint32_t P, T prod) {
     switch (R) {
       SG_TRIE_CASE(0) SG_TRIE_CASE(1) SG_TRIE_CASE(2) SG_TRIE_CASE(3)
       SG_TRIE_CASE(4) SG_TRIE_CASE(5) SG_TRIE_CASE(6) SG_TRIE_CASE(7)
@@ -152,33 +250,28 @@ struct Trie {
   }
 #undef SG_TRIE_CASE
 
-  // ------------------------------------------------------- outer trie levels
-  // Dimension t (D-1 .. I), ascending l_t (Alg. 3 order); `budget` is what is
-  // left for dimensions t..0, sigma = sum_{u>t} l_u (the shift of dimension
-  // t's digit), P = the digits of dimensions > t, prod = their hat product.
+  // node at dimension t >= I with run-time budget B (levels of dimensions
+  // t..0 sum to B): a run-time loop over l_t, each child inlined once
   template <int J, int t>
-  static __device__ __forceinline__ void outer(Ctx& c, int budget, int sigma, uint32_t P, T prod) {
-    if constexpr (O == 0) {
-      block<J, J>(c, 0u, T(1));  // no outer dimensions: one block per group
-    } else if constexpr (t < I) {
-      leaf<J>(c, budget, sigma, P, prod);
-    } else if constexpr (t == I) {
-      for (int lt = 0; lt <= budget; ++lt) {
+  static __device__ __forceinline__ void node(Ctx& c, int B, uint32_t P, T prod) {
+    if (B <= flat_max<t>()) {
+      flat_dispatch<J, t>(c, B, P, prod);
+      return;
+    }
+    const int SG = J - B;  // shift of dimension t's digit
+    if constexpr (t == I) {
+      for (int lt = 0; lt < B - kTail; ++lt) {
         const T ph = c.phs[(SM_IN + lt) * NT];
-        const uint32_t kt = c.K[t] >> (NM - 1 - lt);
-        outer<J, t - 1>(c, budget - lt, sigma + lt, P | (kt << sigma), prod * ph);
+        const uint32_t kt = c.K[I] >> (NM - 1 - lt);
+        leaf<J>(c, B - lt, P | (kt << SG), prod * ph);
       }
+      inner_tail<J, kTail>(c, B, P, prod);
     } else {
-      T u = c.xs[(t - I - 1) * NT];  // u_l = 2^l x - k_t(l), starting at l = 0
-      for (int lt = 0; lt <= budget; ++lt) {
-        const T w = T(1) - u;
-        const T mn = u < w ? u : w;
-        T ph = mn + mn;
-        ph = ph > T(0) ? ph : T(0);
+      T u = c.xs[(t - I - 1) * NT];
+      for (int lt = 0; lt <= B; ++lt) {
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
-        outer<J, t - 1>(c, budget - lt, sigma + lt, P | (kt << sigma), prod * ph);
-        u = u + u;
-        u = u >= T(1) ? u - T(1) : u;
+        node<J, t - 1>(c, B - lt, P | (kt << SG), prod * hat_u(u));
+        u = dbl_u(u);
       }
     }
   }
@@ -187,7 +280,8 @@ struct Trie {
   static __device__ __forceinline__ void groups(Ctx& c, int n) {
     if constexpr (J <= J1 && J < NM) {
       if (J < n) {
-        outer<J, D - 1>(c, J, 0, 0u, T(1));
+        if constexpr (O == 0) block<J, J>(c, 0u, T(1));  // no outer dimensions: one block per group
+        else node<J, D - 1>(c, J, 0u, T(1));
         groups<J + 1, J1>(c, n);
       }
     }
