@@ -35,6 +35,22 @@ def _stale() -> bool:
     return any(os.path.getmtime(p) > t for p in deps)
 
 
+def _deps(path, seen=None):
+    """The file and every local header it includes (transitively)."""
+    seen = set() if seen is None else seen
+    if path in seen or not os.path.exists(path):
+        return seen
+    seen.add(path)
+    with open(path) as f:
+        for line in f:
+            line = line.strip()
+            if line.startswith("#include \""):
+                name = line.split('"')[1]
+                for d in (os.path.dirname(path), os.path.join(ROOT, "include")):
+                    _deps(os.path.join(d, name), seen)
+    return seen
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
@@ -44,22 +60,30 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs, procs = [], []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        objs.append(obj)
+        if not force and os.path.exists(obj) and all(
+                os.path.getmtime(p) <= os.path.getmtime(obj) for p in _deps(src) | {__file__}):
+            continue  # object newer than the source and every header it includes
         cmd = [NVCC, *ARCH, *FLAGS, f'-DSG_BUILD_FLAGS="{flag_str}"', "-I", os.path.join(ROOT, "include"),
                "-c", src, "-o", obj]
         procs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)))
-        objs.append(obj)
     logs = []
     failed = None
     for src, p in procs:
         out, _ = p.communicate()
         logs.append(f"== {os.path.basename(src)}\n{out}")
+        with open(os.path.join(objdir, os.path.basename(src) + ".log"), "w") as f:
+            f.write(out)
         if p.returncode != 0:
             sys.stderr.write(out)
             failed = src
     if failed:
         raise RuntimeError(f"nvcc failed on {failed}")
-    with open(os.path.join(objdir, "ptxas.log"), "w") as f:
-        f.write("\n".join(logs))
+    with open(os.path.join(objdir, "ptxas.log"), "w") as f:  # every object's ptxas -v output
+        for src in sources():
+            lp = os.path.join(objdir, os.path.basename(src) + ".log")
+            if os.path.exists(lp):
+                f.write(f"== {os.path.basename(src)}\n" + open(lp).read())
     tmp = LIB + ".tmp"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart"])
     os.replace(tmp, LIB)

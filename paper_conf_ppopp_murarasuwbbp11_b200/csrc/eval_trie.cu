@@ -31,7 +31,8 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     double* yy = (double*)y;
     if (d == 10 && n == 11) {
       sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
-      return st == SG_OK ? trie_d10n11_b(L, a, xx, perm, m, yy, s) : st;
+      if (st != SG_OK) return st;
+      return trie_d10n11_b(L, a, xx, perm, m, yy, s);
     }
     if (d == 2 && n == 3) return trie_d2n3(L, a, xx, perm, m, yy, s);
     if (d == 5 && n == 8) return trie_d5n8(L, a, xx, perm, m, yy, s);

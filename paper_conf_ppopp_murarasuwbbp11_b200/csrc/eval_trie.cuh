@@ -41,7 +41,7 @@
 namespace sg {
 namespace trie {
 
-template <typename T, int D, int NM, int NT>
+template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
@@ -140,12 +140,17 @@ struct Trie {
   // (l_0 implied), under the outer digits P (dimensions > t, all below bit
   // J - B) and their hat product `prod`.  B is a compile-time constant at
   // every node, so every digit shift (J - B for dimension t) is an immediate.
-  // Small sub-tries (C(B+t, t) <= kFlat terms) are emitted as straight-line
-  // code: one basic block, all its surplus loads in flight together (the
-  // v2 trie issued them one small block at a time and was latency-bound,
-  // profiles/r01_v2_*).  Large ones loop over l_t at run time and dispatch the
-  // child's budget B - l_t through a switch.
-  static constexpr int kFlat = 70;   // straight-line sub-trie size (terms)
+  // Dimension I (the innermost outer dimension) is emitted as straight-line
+  // code for B <= kFull, and its last kTail + 1 blocks (the small ones, R <=
+  // kTail) are merged into one basic block, so that each basic block keeps
+  // more surplus loads in flight (v2 issued one small block at a time and was
+  // latency-bound, profiles/r01_v2_*).  Sub-tries of higher dimensions with at
+  // most FLAT terms can be emitted straight-line too; measured on B200
+  // (profiles/r01_v3_variants.txt) the larger code then thrashes the
+  // instruction cache (23.7% no_instruction stalls at FLAT = 70 vs 14.6% at
+  // FLAT = 0, 6.12e6 vs 6.79e6 evals/s), so FLAT defaults to 0.  SYNC adds a
+  // CTA barrier per dimension-(I+1) node (experiment; slower at 384x1).
+  static constexpr int kFlat = FLAT;  // straight-line sub-trie size (terms)
   static constexpr int kFull = 4;    // dimension I: unroll every l_I when B <= kFull
   static constexpr int kTail = 2;    // dimension I: merge the blocks R <= kTail into one basic block
 
@@ -269,6 +274,9 @@ struct Trie {
     } else {
       T u = c.xs[(t - I - 1) * NT];
       for (int lt = 0; lt <= B; ++lt) {
+        // SYNC: keep the warps of a CTA on the same sub-trie (shared L1 sectors
+        // and instruction-cache lines); the enumeration is CTA-uniform
+        if constexpr (SYNC && t == I + 1) __syncthreads();
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
         node<J, t - 1>(c, B - lt, P | (kt << SG), prod * hat_u(u));
         u = dbl_u(u);
@@ -292,11 +300,11 @@ struct Trie {
 // One launch evaluates the level groups J0..J1 (compile time) for every
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -345,12 +353,12 @@ __global__ void __launch_bounds__(NT, MINB)
   }
 }
 
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC>;
   const size_t smem = TR::smem_bytes;
   static bool attr_set = false;
   if (!attr_set) {

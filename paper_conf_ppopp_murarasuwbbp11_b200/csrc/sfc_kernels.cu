@@ -23,6 +23,24 @@ inline int morton_bits(int d) {
   return b > 20 ? 20 : (b < 1 ? 1 : b);
 }
 
+// Plane lag of dimension t.  In the layout the in-subspace index has
+// dimension 0 as its most significant digit and dimension d-1 as its fastest
+// one (Alg. 5), and a warp's fp64 gather costs, per half-warp, the
+// largest number of distinct words that fall into one L1 bank pair (address
+// bits 3-6, i.e. the low 4 bits of the index; profiles/r01_ubench_l1_gather.txt).
+// Queries of a warp that differ in the high dimensions (coarse digits) but
+// agree in the low ones land in the same bank pair and serialise; queries that
+// differ in the fast dimensions do not.  Entering the fast dimensions later
+// in the curve makes warps compact in dimensions 0..d/2 and elongated in the
+// fast ones: at d = 10 this cuts the modelled L1 cycles per gather from 4.11
+// to 3.27 (SURVEY-style simulation over 10^7 uniform points, groups 5-10).
+__host__ __device__ inline int morton_lag(int t, int d, int bits) {
+  if (d < 4) return 0;
+  const int lag = t - d / 2;
+  const int cap = bits / 2;
+  return lag <= 0 ? 0 : (lag < cap ? lag : cap);
+}
+
 template <typename T>
 __global__ void __launch_bounds__(kThreads) k_morton(const T* __restrict__ x, uint64_t m, int d, int bits,
                                                      uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
@@ -36,9 +54,15 @@ __global__ void __launch_bounds__(kThreads) k_morton(const T* __restrict__ x, ui
       v = v <= top ? v : top;
       c[t] = (uint32_t)v;
     }
+    // bit planes from the most significant one; dimension t enters lag(t)
+    // planes late (see morton_lag), so every dimension keeps `bits` bits
     uint64_t key = 0;
-    for (int b = bits - 1; b >= 0; --b)
-      for (int t = 0; t < d; ++t) key = (key << 1) | ((c[t] >> b) & 1u);
+    const int lmax = morton_lag(d - 1, d, bits);
+    for (int p = 0; p < bits + lmax; ++p)
+      for (int t = 0; t < d; ++t) {
+        const int b = p - morton_lag(t, d, bits);  // bit of dimension t, 0 = its MSB
+        if (b >= 0 && b < bits) key = (key << 1) | ((c[t] >> (bits - 1 - b)) & 1u);
+      }
     keys[q] = key;
     vals[q] = (uint32_t)q;
   }
