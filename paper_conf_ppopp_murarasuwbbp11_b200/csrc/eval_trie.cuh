@@ -62,24 +62,26 @@ struct Trie {
     uint32_t b;  // running subspace base (elements), warp-uniform
   };
 
-  static constexpr uint32_t cnt(int R) {  // subspaces per block = C(R+I-1, I-1)
+  static constexpr uint32_t cnt(int R, int NI) {  // subspaces per block = C(R+NI-1, NI-1)
     uint32_t c = 1;
-    for (int k = 1; k <= I - 1; ++k) c = c * (uint32_t)(R + k) / (uint32_t)k;
+    for (int k = 1; k <= NI - 1; ++k) c = c * (uint32_t)(R + k) / (uint32_t)k;
     return c;
   }
 
   // ---------------------------------------------------------------- leaf block
   // Group J, R = J - sigma: every shift below is a compile-time constant.
-  template <int J, int R>
+  // The block spans the NI innermost dimensions (NI = I, or I - 1 for the
+  // pieces of a split block, whose dimension-(NI) digit is then in P).
+  template <int J, int R, int NI = I>
   static __device__ __forceinline__ void block(Ctx& c, uint32_t P, T prod) {
     constexpr int SG = J - R;  // sigma = sum of the outer levels
     // per-lane block base &alpha[b + P] (P = the outer digits, all below bit SG)
     const T* base = c.alpha + c.b + P;
     uint32_t k0, k1, k2, k3;  // opaque copies: keep the per-block cell work inside the trie
     asm volatile("mov.b32 %0, %1;" : "=r"(k0) : "r"(c.K[0]));
-    asm volatile("mov.b32 %0, %1;" : "=r"(k1) : "r"(c.K[I > 1 ? 1 : 0]));
-    asm volatile("mov.b32 %0, %1;" : "=r"(k2) : "r"(c.K[I > 2 ? 2 : 0]));
-    asm volatile("mov.b32 %0, %1;" : "=r"(k3) : "r"(c.K[I > 3 ? 3 : 0]));
+    asm volatile("mov.b32 %0, %1;" : "=r"(k1) : "r"(c.K[NI > 1 ? 1 : 0]));
+    asm volatile("mov.b32 %0, %1;" : "=r"(k2) : "r"(c.K[NI > 2 ? 2 : 0]));
+    asm volatile("mov.b32 %0, %1;" : "=r"(k3) : "r"(c.K[NI > 3 ? 3 : 0]));
     // C'[s] = (k_0(R-s) << (s+SG)) | (k_1 digits at level s, shifted by SG);
     // bits below SG are garbage and cleared by every row mask.
     const uint32_t K0J = k0 >> (NM - 1 - J);
@@ -87,32 +89,32 @@ struct Trie {
 #pragma unroll
     for (int s = 0; s <= R; ++s) {
       const uint32_t hi = K0J & ~((1u << (s + SG)) - 1u);
-      const uint32_t lo = (I > 1) ? (k1 >> (NM - 1 - s - SG)) : 0u;
+      const uint32_t lo = (NI > 1) ? (k1 >> (NM - 1 - s - SG)) : 0u;
       Cs[s] = hi | lo;
     }
     // hat values of dimensions 2, 3 for levels 0..R, from shared memory
     T ph2[R + 1], ph3[R + 1];
 #pragma unroll
     for (int l = 0; l <= R; ++l) {
-      ph2[l] = (I >= 3) ? c.phs[(0 * NM + l) * NT] : T(1);
-      ph3[l] = (I >= 4) ? c.phs[(1 * NM + l) * NT] : T(1);
+      ph2[l] = (NI >= 3) ? c.phs[(0 * NM + l) * NT] : T(1);
+      ph3[l] = (NI >= 4) ? c.phs[(1 * NM + l) * NT] : T(1);
     }
-    constexpr int R3 = (I >= 4) ? R : 0;
+    constexpr int R3 = (NI >= 4) ? R : 0;
     T acc = T(0);
     int cidx = 0;  // compile-time after unrolling: rank of the term inside the block
 #pragma unroll
     for (int l3 = 0; l3 <= R3; ++l3) {
       // k_3(l3) << SG
-      const uint32_t X3 = (I >= 4) ? ((k3 >> (NM - 1 - l3 - SG)) & ~((1u << SG) - 1u)) : 0u;
-      const int R2 = (I >= 3) ? R - l3 : 0;
+      const uint32_t X3 = (NI >= 4) ? ((k3 >> (NM - 1 - l3 - SG)) & ~((1u << SG) - 1u)) : 0u;
+      const int R2 = (NI >= 3) ? R - l3 : 0;
       T acc3 = T(0);
 #pragma unroll
       for (int l2 = 0; l2 <= R2; ++l2) {
         // X_row = (k_2(l2) << (l3+SG)) | X3
-        uint32_t Xr = (I >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG)) & ~((1u << (l3 + SG)) - 1u)) | X3) : X3;
+        uint32_t Xr = (NI >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG)) & ~((1u << (l3 + SG)) - 1u)) | X3) : X3;
         asm("mov.b32 %0, %0;" : "+r"(Xr));
         const uint32_t M = 0xffffffffu << (l2 + l3 + SG);
-        const int R1 = (I >= 2) ? R - l3 - l2 : 0;
+        const int R1 = (NI >= 2) ? R - l3 - l2 : 0;
         T acc2 = T(0);
 #pragma unroll
         for (int l1 = 0; l1 <= R1; ++l1) {
@@ -123,16 +125,16 @@ struct Trie {
           const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
           asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
           const T a = __ldg(p + ((uint32_t)cidx << J));
-          if (I >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[I > 1 ? 1 : 0][l1], acc2);
+          if (NI >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[NI > 1 ? 1 : 0][l1], acc2);
           else acc2 = fma(a, c.ph[0][l0], acc2);
           ++cidx;
         }
-        acc3 = (I >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
+        acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
       }
-      acc = (I >= 4) ? fma(acc3, ph3[l3], acc) : acc3;
+      acc = (NI >= 4) ? fma(acc3, ph3[l3], acc) : acc3;
     }
     c.res = fma(acc, prod, c.res);
-    c.b += cnt(R) << J;
+    c.b += cnt(R, NI) << J;
   }
 
   // ------------------------------------------------------- outer trie levels
@@ -239,9 +241,59 @@ struct Trie {
     }
   }
 
+  // Blocks of I = 4 dimensions with R >= kSplit (84+ terms, 24% of the terms
+  // of group 10 but 89% of its block code) are split along dimension 3 into
+  // 3-dimensional pieces shared by every R: l_3 runs at run time, the piece
+  // for budget R - l_3 is dispatched by a switch, and the last kTail3 + 1
+  // (small) pieces are merged into one basic block.  Subspace order is kept:
+  // l_3 is the slowest of dimensions 0..3 (Alg. 3).
+  static constexpr int kSplit = 6;
+  static constexpr int kTail3 = 2;
+
+#define SG_TRIE_CASE3(r) \
+  case r:                \
+    if constexpr (r <= J) block<J, (r <= J ? r : 0), 3>(c, P, prod); \
+    break;
+  template <int J>
+  static __device__ __forceinline__ void leaf3(Ctx& c, int R, uint32_t P, T prod) {
+    switch (R) {
+      SG_TRIE_CASE3(0) SG_TRIE_CASE3(1) SG_TRIE_CASE3(2) SG_TRIE_CASE3(3)
+      SG_TRIE_CASE3(4) SG_TRIE_CASE3(5) SG_TRIE_CASE3(6) SG_TRIE_CASE3(7)
+      SG_TRIE_CASE3(8) SG_TRIE_CASE3(9) SG_TRIE_CASE3(10) SG_TRIE_CASE3(11)
+      SG_TRIE_CASE3(12) SG_TRIE_CASE3(13) SG_TRIE_CASE3(14) SG_TRIE_CASE3(15)
+      default: break;
+    }
+  }
+#undef SG_TRIE_CASE3
+
+  // pieces l_3 = R - RT .. R of a split block (compile-time), one basic block
+  template <int J, int R, int RT>
+  static __device__ __forceinline__ void tail3(Ctx& c, uint32_t P, T prod) {
+    if constexpr (RT >= 0) {
+      constexpr int l3 = R - RT;
+      const T ph = c.phs[(1 * NM + l3) * NT];
+      const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
+      block<J, RT, 3>(c, P | (k3 << (J - R)), prod * ph);
+      tail3<J, R, RT - 1>(c, P, prod);
+    }
+  }
+
+  template <int J, int R>
+  static __device__ __forceinline__ void split4(Ctx& c, uint32_t P, T prod) {
+    for (int l3 = 0; l3 < R - kTail3; ++l3) {
+      const T ph = c.phs[(1 * NM + l3) * NT];
+      const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
+      leaf3<J>(c, R - l3, P | (k3 << (J - R)), prod * ph);
+    }
+    tail3<J, R, kTail3>(c, P, prod);
+  }
+
 #define SG_TRIE_CASE(r) \
   case r:               \
-    if constexpr (r <= J) block<J, (r <= J ? r : 0)>(c, P, prod); \
+    if constexpr (r <= J) {                                        \
+      if constexpr (I == 4 && r >= kSplit) split4<J, (r <= J ? r : 0)>(c, P, prod); \
+      else block<J, (r <= J ? r : 0)>(c, P, prod);                 \
+    }                                                              \
     break;
   template <int J>
   static __device__ __forceinline__ void leaf(Ctx& c, int R, uint32_t P, T prod) {
