@@ -241,13 +241,14 @@ struct Trie {
     }
   }
 
-  // Blocks of I = 4 dimensions with R >= kSplit (84+ terms, 24% of the terms
-  // of group 10 but 89% of its block code) are split along dimension 3 into
-  // 3-dimensional pieces shared by every R: l_3 runs at run time, the piece
-  // for budget R - l_3 is dispatched by a switch, and the last kTail3 + 1
-  // (small) pieces are merged into one basic block.  Subspace order is kept:
-  // l_3 is the slowest of dimensions 0..3 (Alg. 3).
-  static constexpr int kSplit = 6;
+  // Blocks of I = 4 dimensions with R >= kSplit can be split along dimension
+  // 3 into 3-dimensional pieces shared by every R (l_3 at run time, the piece
+  // for budget R - l_3 dispatched by a switch, the last kTail3 + 1 pieces
+  // merged; subspace order kept: l_3 is the slowest of dimensions 0..3, Alg. 3,
+  // P:L373).  This shrinks the code (instruction-cache stalls 4.3% -> 1.6%) but
+  // the smaller basic blocks keep fewer loads in flight: measured at kSplit = 6
+  // 5.99e6 vs 6.70e6 evals/s (profiles/r01_v3_variants.txt), so it is off.
+  static constexpr int kSplit = 16;
   static constexpr int kTail3 = 2;
 
 #define SG_TRIE_CASE3(r) \
