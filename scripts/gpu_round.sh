@@ -22,7 +22,7 @@ timeout 300 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_d
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > gpurun_out/${TAG}_traffic.log 2>&1
 python scripts/ncu_traffic.py gpurun_out/${TAG}_traffic.csv 10000000 > gpurun_out/${TAG}_eval_kernel_ncu.json 2>&1
 timeout 420 ncu --set full --clock-control none --import-source on -k regex:k_eval_trie --launch-skip 4 -c 1 -o /tmp/${TAG}_eval \
-  python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > gpurun_out/${TAG}_ncu_eval.log 2>&1
+  python bench.py --steps 1 --warmup 0 --m 1000000 --no-e2e --no-cpu > gpurun_out/${TAG}_ncu_eval.log 2>&1
 timeout 120 python scripts/ncu_summary.py /tmp/${TAG}_eval.ncu-rep > gpurun_out/${TAG}_eval_ncu.txt 2>&1
 timeout 120 ncu -i /tmp/${TAG}_eval.ncu-rep --page source --csv --print-source sass > /tmp/${TAG}_src.csv 2>/dev/null
 timeout 120 python scripts/ncu_mix.py /tmp/${TAG}_src.csv > gpurun_out/${TAG}_eval_mix.txt 2>&1
