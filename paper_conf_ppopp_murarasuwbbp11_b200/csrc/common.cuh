@@ -11,6 +11,11 @@ struct sg_grid_s {
   sg::Layout L;         // host tables
   int device;           // device that was current at sg_create
   sg::Layout* d_L;      // device copy of L
+  // pole-family tables of the hierarchization (built on first use, per device
+  // copy of the grid; hier_kernels.cu): per dimension, per family a packed
+  // (|l_{-t}|, suffix sum) word and the offset of its first block base, and
+  // per family per block the global offset of the block
+  void* d_hier_tab = nullptr;
 };
 
 namespace sg {

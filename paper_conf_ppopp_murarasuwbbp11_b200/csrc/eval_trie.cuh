@@ -41,7 +41,7 @@
 namespace sg {
 namespace trie {
 
-template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false>
+template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
@@ -144,7 +144,8 @@ struct Trie {
   // every node, so every digit shift (J - B for dimension t) is an immediate.
   // Dimension I (the innermost outer dimension) is emitted as straight-line
   // code for B <= kFull, and its last kTail + 1 blocks (the small ones, R <=
-  // kTail) are merged into one basic block, so that each basic block keeps
+  // kTail: 1 + 4 + 10 + 20 terms) are merged into one basic block (kTail = 3
+  // measured 2.8% faster than 2), so that each basic block keeps
   // more surplus loads in flight (v2 issued one small block at a time and was
   // latency-bound, profiles/r01_v2_*).  Sub-tries of higher dimensions with at
   // most FLAT terms can be emitted straight-line too; measured on B200
@@ -154,7 +155,7 @@ struct Trie {
   // CTA barrier per dimension-(I+1) node (experiment; slower at 384x1).
   static constexpr int kFlat = FLAT;  // straight-line sub-trie size (terms)
   static constexpr int kFull = 4;    // dimension I: unroll every l_I when B <= kFull
-  static constexpr int kTail = 2;    // dimension I: merge the blocks R <= kTail into one basic block
+  static constexpr int kTail = TAIL;  // dimension I: merge the blocks R <= kTail into one basic block
 
   static constexpr uint32_t binom(int a, int b) {
     uint32_t c = 1;
@@ -353,11 +354,11 @@ struct Trie {
 // One launch evaluates the level groups J0..J1 (compile time) for every
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -406,12 +407,12 @@ __global__ void __launch_bounds__(NT, MINB)
   }
 }
 
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL>;
   const size_t smem = TR::smem_bytes;
   static bool attr_set = false;
   if (!attr_set) {

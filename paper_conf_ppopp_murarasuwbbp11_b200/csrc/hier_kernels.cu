@@ -59,67 +59,125 @@ __device__ bool family_levels(const Layout& L, int t, uint64_t f, int32_t* lv) {
   return true;
 }
 
+// ---- v2: family tables built once per grid (first call), so a family's CTA
+// needs no serial set-up (v1: thread 0 unranked the family and ranked its L
+// blocks while 255 threads waited at a barrier, after copying the 8.6 KB
+// Layout into shared memory -- 47% barrier stalls, profiles/r01_v3_hier_ncu.txt).
+//
+// Per dimension t and family f: info[2f] = |l_{-t}| | (sum_{u>t} l_u) << 8,
+// info[2f+1] = index of the family's first block base in `base`, and
+// base[first + k] = global offset of the family's block with l_t = k.
+// One CTA per family loads the family into shared memory (block by block,
+// coalesced), then computes every l_t >= 1 point from its two 1D parents
+// (Alg. 1 / Alg. 6) and writes it back.
+struct HierTab {
+  uint64_t F;          // families per dimension (|l_{-t}| <= n-2)
+  uint64_t nbase;      // block bases per dimension (= number of subspaces with |l_{-t}| <= n-2)
+  uint32_t* info;      // [d][F][2]
+  uint64_t* base;      // [d][nbase]
+};
+
+template <int DUMMY = 0>
+__global__ void __launch_bounds__(kThreads) k_hier_table(const Layout* __restrict__ gL, int t, uint64_t F,
+                                                         uint32_t* __restrict__ info, uint64_t* __restrict__ base) {
+  const Layout& L = *gL;
+  const uint64_t f = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (f >= F) return;
+  int32_t lv[SG_MAX_D];
+  family_levels(L, t, f, lv);
+  int s = 0, suf = 0;
+  for (int u = 0; u < L.d; ++u) {
+    s += lv[u];
+    if (u > t) suf += lv[u];
+  }
+  // first = sum over the families before f of their block counts n - s':
+  // families are ordered by s' (|L^{d-1}_{s'}| = C(s'+d-2, d-2) of them), then in Alg. 3 order
+  const int dm = L.d - 1;
+  uint64_t first = 0, before = 0;
+  for (int sp = 0; sp < s; ++sp) {
+    const uint64_t c = dm == 0 ? (sp == 0 ? 1 : 0) : L.C(dm - 1, sp);
+    first += c * (uint64_t)(L.n - sp);
+    before += c;
+  }
+  first += (f - before) * (uint64_t)(L.n - s);
+  info[2 * f] = (uint32_t)s | ((uint32_t)suf << 8);
+  info[2 * f + 1] = (uint32_t)first;
+  for (int k = 0; k < L.n - s; ++k) {
+    lv[t] = k;
+    const int j = s + k;
+    base[first + k] = L.off[j] + (subspace_rank(L, lv) << j);
+  }
+}
+
 template <typename T>
-__global__ void __launch_bounds__(kThreads) k_hier_family(const Layout* __restrict__ gL, int t, T* __restrict__ v) {
+__global__ void __launch_bounds__(kThreads) k_hier_family2(int n, const uint32_t* __restrict__ info,
+                                                           const uint64_t* __restrict__ bases, T* __restrict__ v) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* fam = reinterpret_cast<T*>(smem_raw);
-  __shared__ FamilyInfo fi;
-  __shared__ Layout sL;
-  {
-    const uint32_t* src = reinterpret_cast<const uint32_t*>(gL);
-    uint32_t* dst = reinterpret_cast<uint32_t*>(&sL);
-    for (int k = threadIdx.x; k < (int)(sizeof(Layout) / 4); k += blockDim.x) dst[k] = src[k];
-  }
+  __shared__ uint64_t base[SG_MAX_N];
+  const uint32_t w0 = __ldg(info + 2 * blockIdx.x), first = __ldg(info + 2 * blockIdx.x + 1);
+  const int s = (int)(w0 & 0xff), suf = (int)(w0 >> 8), L = n - s;
+  if ((int)threadIdx.x < L) base[threadIdx.x] = __ldg(bases + first + threadIdx.x);
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int32_t lv[SG_MAX_D];
-    family_levels(sL, t, blockIdx.x, lv);
-    int s = 0, suf = 0;
-    for (int u = 0; u < sL.d; ++u) {
-      s += lv[u];
-      if (u > t) suf += lv[u];
-    }
-    fi.s = s;
-    fi.suf = suf;
-    fi.L = sL.n - s;
-    for (int k = 0; k < fi.L; ++k) {
-      lv[t] = k;
-      int j = s + k;
-      fi.base[k] = sL.off[j] + (subspace_rank(sL, lv) << j);
-    }
-  }
-  __syncthreads();
-  const int s = fi.s, L = fi.L, suf = fi.suf;
   const uint32_t E = ((1u << L) - 1u) << s;  // family size 2^s (2^L - 1)
-  // load: element e lies in block k = floor(log2((e >> s) + 1))
-  for (uint32_t e = threadIdx.x; e < E; e += blockDim.x) {
-    int k = 31 - __clz((e >> s) + 1);
-    uint32_t w = e - (((1u << k) - 1u) << s);
-    fam[e] = v[fi.base[k] + w];
+  // load block by block: block k holds 2^(s+k) consecutive values (coalesced)
+  for (int k = 0; k < L; ++k) {
+    const uint32_t sz = 1u << (s + k), o = ((1u << k) - 1u) << s;
+    const T* src = v + base[k];
+    for (uint32_t w = threadIdx.x; w < sz; w += blockDim.x) fam[o + w] = src[w];
   }
   __syncthreads();
   const uint32_t lomask = (1u << suf) - 1u;
-  for (uint32_t e = (1u << s) + threadIdx.x; e < E; e += blockDim.x) {  // blocks k >= 1
-    int k = 31 - __clz((e >> s) + 1);
-    uint32_t w = e - (((1u << k) - 1u) << s);
-    uint32_t lo = w & lomask;
-    uint32_t c = (w >> suf) & ((1u << k) - 1u);
-    uint32_t hi = w >> (suf + k);
-    T vl = T(0), vr = T(0);
-    if (c != 0) {  // left parent at c / 2^k
-      int b = __ffs(c) - 1;
-      int kp = k - 1 - b;
-      uint32_t cp = (c >> b) >> 1;
-      vl = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
+  for (int k = 1; k < L; ++k) {  // blocks k >= 1 change; parents live in blocks < k
+    const uint32_t sz = 1u << (s + k), o = ((1u << k) - 1u) << s;
+    T* dst = v + base[k];
+    for (uint32_t w = threadIdx.x; w < sz; w += blockDim.x) {
+      const uint32_t lo = w & lomask;
+      const uint32_t c = (w >> suf) & ((1u << k) - 1u);
+      const uint32_t hi = w >> (suf + k);
+      T vl = T(0), vr = T(0);
+      if (c != 0) {  // left parent at c / 2^k
+        const int b = __ffs(c) - 1;
+        const int kp = k - 1 - b;
+        const uint32_t cp = (c >> b) >> 1;
+        vl = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
+      }
+      if (c + 1 != (1u << k)) {  // right parent at (c+1) / 2^k
+        const int b = __ffs(c + 1) - 1;
+        const int kp = k - 1 - b;
+        const uint32_t cp = ((c + 1) >> b) >> 1;
+        vr = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
+      }
+      dst[w] = fam[o + w] - (vl + vr) / T(2);
     }
-    if (c + 1 != (1u << k)) {  // right parent at (c+1) / 2^k
-      int b = __ffs(c + 1) - 1;
-      int kp = k - 1 - b;
-      uint32_t cp = ((c + 1) >> b) >> 1;
-      vr = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
-    }
-    v[fi.base[k] + w] = fam[e] - (vl + vr) / T(2);
   }
+  (void)E;
+}
+
+sg_status hier_table(sg_grid_s* g, HierTab* tab, cudaStream_t s) {
+  const Layout& L = g->L;
+  const int d = L.d, n = L.n;
+  tab->F = (d == 1) ? 1 : L.C(d - 1, n - 2);
+  // block bases per dimension: sum over families of n - |l_{-t}|
+  uint64_t nb = 0;
+  for (int sp = 0; sp <= n - 2; ++sp) nb += (d == 1 ? (sp == 0 ? 1 : 0) : L.C(d - 2, sp)) * (uint64_t)(n - sp);
+  tab->nbase = nb;
+  if (!g->d_hier_tab) {
+    const size_t bytes = (size_t)d * (tab->F * 2 * sizeof(uint32_t) + nb * sizeof(uint64_t));
+    cudaError_t e = cudaMalloc(&g->d_hier_tab, bytes);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(hierarchization tables)");
+    uint64_t* b = (uint64_t*)g->d_hier_tab;
+    uint32_t* in = (uint32_t*)(b + (size_t)d * nb);
+    for (int t = 0; t < d; ++t) {
+      const unsigned blocks = (unsigned)((tab->F + kThreads - 1) / kThreads);
+      k_hier_table<<<blocks, kThreads, 0, s>>>(g->d_L, t, tab->F, in + (size_t)t * tab->F * 2, b + (size_t)t * nb);
+      sg_status st = launched("k_hier_table");
+      if (st != SG_OK) return st;
+    }
+  }
+  tab->base = (uint64_t*)g->d_hier_tab;
+  tab->info = (uint32_t*)(tab->base + (size_t)d * nb);
+  return SG_OK;
 }
 
 // Fallback for families larger than shared memory: one thread per point,
@@ -170,15 +228,17 @@ sg_status hierarchize_t(const sg_grid_s* g, T* v, cudaStream_t s) {
   cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   const size_t static_smem = sizeof(Layout) + sizeof(FamilyInfo) + 64;
   if (fam_bytes + static_smem <= (size_t)max_smem) {
-    cudaError_t e = cudaFuncSetAttribute(k_hier_family<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    HierTab tab;
+    sg_status st = hier_table(const_cast<sg_grid_s*>(g), &tab, s);
+    if (st != SG_OK) return st;
+    cudaError_t e = cudaFuncSetAttribute(k_hier_family2<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)fam_bytes);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_hier_family)");
-    // families with |l_{-t}| <= n-2: sum_{s<=n-2} C(s+d-2, d-2) = C(n-2+d-1, d-1)
-    uint64_t F = (d == 1) ? 1 : L.C(d - 1, n - 2);
-    if (F > 0x7fffffffull) return SG_ERR_OVERFLOW;
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_hier_family2)");
+    if (tab.F > 0x7fffffffull) return SG_ERR_OVERFLOW;
     for (int t = 0; t < d; ++t) {
-      k_hier_family<T><<<(unsigned)F, kThreads, fam_bytes, s>>>(g->d_L, t, v);
-      sg_status st = launched("k_hier_family");
+      k_hier_family2<T><<<(unsigned)tab.F, kThreads, fam_bytes, s>>>(n, tab.info + (size_t)t * tab.F * 2,
+                                                                       tab.base + (size_t)t * tab.nbase, v);
+      st = launched("k_hier_family2");
       if (st != SG_OK) return st;
     }
     return SG_OK;

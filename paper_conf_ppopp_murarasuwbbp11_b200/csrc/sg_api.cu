@@ -176,6 +176,7 @@ sg_status sg_destroy(sg_grid g) {
     DeviceGuard guard(g->device);
     cudaDeviceSynchronize();
     cudaFree(g->d_L);
+    if (g->d_hier_tab) cudaFree(g->d_hier_tab);
   }
   delete g;
   return SG_OK;
