@@ -41,13 +41,21 @@
 namespace sg {
 namespace trie {
 
-template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3>
+template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
+          int CHUNK = 0>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
   // shared memory, [row][lane]: hat values of dimensions 2, 3 (loaded per
   // block), of dimension I (per outer node), then x of dimensions I+1..D-1
-  static constexpr int SM_IN = 2 * NM;
+  // HREG: hat values of dimensions 2, 3 recomputed per block by exact
+  // doubling from x (registers) instead of loaded from shared memory (LDS
+  // use the same L1 data stage as the surplus gathers).  Experiment, off:
+  // ptxas then keeps 4 instead of 13 loads in flight (4.88e6 vs 6.91e6).
+  // CHUNK > 0: two-phase blocks (loads of CHUNK terms, then their Horner
+  // accumulation).  Experiment, off: 15 vs 13 loads in flight at first use
+  // in SASS, but no measurable change (6.87e6 vs 6.91e6 evals/s).
+  static constexpr int SM_IN = HREG ? 0 : 2 * NM;
   static constexpr int SM_PH = O > 0 ? NM : 0;
   static constexpr int SM_X = O > 1 ? O - 1 : 0;
   static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X) * NT * sizeof(T);
@@ -57,6 +65,7 @@ struct Trie {
     const T* phs;  // this lane's column of the hat tables (dims 2, 3, I)
     const T* xs;   // this lane's column of the x table of dimensions > I
     T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
+    T xin[2];                 // HREG: x of dimensions 2, 3
     uint32_t K[D];
     T res;
     uint32_t b;  // running subspace base (elements), warp-uniform
@@ -66,6 +75,73 @@ struct Trie {
     uint32_t c = 1;
     for (int k = 1; k <= NI - 1; ++k) c = c * (uint32_t)(R + k) / (uint32_t)k;
     return c;
+  }
+
+  // flat term index of a block -> l3 | l2 << 8 | l1 << 16 (subspace order, l3 slowest)
+  static constexpr int dec(int R, int NI, int ci) {
+    int l3 = 0;
+    if (NI >= 4)
+      while (ci >= (int)cnt(R - l3, 3)) { ci -= (int)cnt(R - l3, 3); ++l3; }
+    int l2 = 0;
+    if (NI >= 3)
+      while (ci >= R - l3 - l2 + 1) { ci -= R - l3 - l2 + 1; ++l2; }
+    return l3 | (l2 << 8) | (ci << 16);
+  }
+  template <int J, int R, int NI, int C0, int I>
+  static __device__ __forceinline__ void chunk_load(const T* base, const uint32_t* Cs, uint32_t k2, uint32_t k3,
+                                                    T (&av)[CHUNK > 0 ? CHUNK : 1]) {
+    constexpr int CNT = (int)cnt(R, NI);
+    if constexpr (I < CHUNK && C0 + I < CNT) {
+      constexpr int code = dec(R, NI, C0 + I);
+      constexpr int l3 = code & 255, l2 = (code >> 8) & 255, l1 = code >> 16;
+      constexpr int SG = J - R;
+      constexpr int s = l1 + l2 + l3;
+      const uint32_t X3 = (NI >= 4) ? ((k3 >> (NM - 1 - l3 - SG)) & ~((1u << SG) - 1u)) : 0u;
+      const uint32_t Xr = (NI >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG)) & ~((1u << (l3 + SG)) - 1u)) | X3) : X3;
+      constexpr uint32_t M = 0xffffffffu << (l2 + l3 + SG);
+      uint32_t V;
+      asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
+      const T* p;
+      asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
+      av[I] = __ldg(p + ((uint32_t)(C0 + I) << J));
+      chunk_load<J, R, NI, C0, I + 1>(base, Cs, k2, k3, av);
+    }
+  }
+  static constexpr bool LAZY = false;  // lazy reads of ph2/ph3 measured no better (ptxas in-flight 13.2 vs 15.1)
+  template <int R, int NI, int C0, int I>
+  static __device__ __forceinline__ void chunk_acc(const Ctx& c, const T* ph2, const T* ph3,
+                                                   const T (&av)[CHUNK > 0 ? CHUNK : 1], T& acc, T& acc2, T& acc3) {
+    constexpr int CNT = (int)cnt(R, NI);
+    if constexpr (I < CHUNK && C0 + I < CNT) {
+      constexpr int code = dec(R, NI, C0 + I);
+      constexpr int l3 = code & 255, l2 = (code >> 8) & 255, l1 = code >> 16;
+      constexpr int l0 = R - l1 - l2 - l3;
+      if constexpr (NI >= 2) acc2 = fma(av[I] * c.ph[0][l0], c.ph[NI > 1 ? 1 : 0][l1], acc2);
+      else acc2 = fma(av[I], c.ph[0][l0], acc2);
+      if constexpr (l1 == ((NI >= 2) ? R - l3 - l2 : 0)) {  // end of row (l3, l2)
+        // hat values of dimensions 2, 3 read at the row / slab end (LAZY) or
+        // from the per-block registers
+        const T h2 = (NI >= 3) ? (LAZY ? c.phs[(0 * NM + l2) * NT] : ph2[l2]) : T(1);
+        acc3 = (NI >= 3) ? fma(acc2, h2, acc3) : acc2;
+        acc2 = T(0);
+        if constexpr (l2 == ((NI >= 3) ? R - l3 : 0)) {  // end of slab l3
+          const T h3 = (NI >= 4) ? (LAZY ? c.phs[(1 * NM + l3) * NT] : ph3[l3]) : T(1);
+          acc = (NI >= 4) ? fma(acc3, h3, acc) : acc3;
+          acc3 = T(0);
+        }
+      }
+      chunk_acc<R, NI, C0, I + 1>(c, ph2, ph3, av, acc, acc2, acc3);
+    }
+  }
+  template <int J, int R, int NI, int C0>
+  static __device__ __forceinline__ void chunks(const Ctx& c, const T* base, const uint32_t* Cs, uint32_t k2,
+                                                uint32_t k3, const T* ph2, const T* ph3, T& acc, T& acc2, T& acc3) {
+    if constexpr (R <= J && C0 < (int)cnt(R, NI)) {  // (R > J only in dead instantiations)
+      T av[CHUNK > 0 ? CHUNK : 1];
+      chunk_load<J, R, NI, C0, 0>(base, Cs, k2, k3, av);
+      chunk_acc<R, NI, C0, 0>(c, ph2, ph3, av, acc, acc2, acc3);
+      chunks<J, R, NI, C0 + CHUNK>(c, base, Cs, k2, k3, ph2, ph3, acc, acc2, acc3);
+    }
   }
 
   // ---------------------------------------------------------------- leaf block
@@ -94,13 +170,33 @@ struct Trie {
     }
     // hat values of dimensions 2, 3 for levels 0..R, from shared memory
     T ph2[R + 1], ph3[R + 1];
+    if constexpr (CHUNK > 0 && LAZY) {
+      // read at the row / slab ends (chunk_acc)
+    } else if constexpr (HREG) {
+      T u2 = c.xin[0], u3 = c.xin[1];
 #pragma unroll
-    for (int l = 0; l <= R; ++l) {
-      ph2[l] = (NI >= 3) ? c.phs[(0 * NM + l) * NT] : T(1);
-      ph3[l] = (NI >= 4) ? c.phs[(1 * NM + l) * NT] : T(1);
+      for (int l = 0; l <= R; ++l) {
+        ph2[l] = (NI >= 3) ? hat_u(u2) : T(1);
+        ph3[l] = (NI >= 4) ? hat_u(u3) : T(1);
+        u2 = dbl_u(u2);
+        u3 = dbl_u(u3);
+      }
+    } else {
+#pragma unroll
+      for (int l = 0; l <= R; ++l) {
+        ph2[l] = (NI >= 3) ? c.phs[(0 * NM + l) * NT] : T(1);
+        ph3[l] = (NI >= 4) ? c.phs[(1 * NM + l) * NT] : T(1);
+      }
     }
-    constexpr int R3 = (NI >= 4) ? R : 0;
     T acc = T(0);
+    if constexpr (CHUNK > 0) {
+      // two phases per chunk of CHUNK terms (flat term index in subspace
+      // order): all loads of the chunk first, then the Horner accumulation,
+      // so that the scheduler keeps the whole chunk of loads in flight
+      T acc2 = T(0), acc3 = T(0);
+      chunks<J, R, NI, 0>(c, base, Cs, k2, k3, ph2, ph3, acc, acc2, acc3);
+    } else {
+    constexpr int R3 = (NI >= 4) ? R : 0;
     int cidx = 0;  // compile-time after unrolling: rank of the term inside the block
 #pragma unroll
     for (int l3 = 0; l3 <= R3; ++l3) {
@@ -132,6 +228,7 @@ struct Trie {
         acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
       }
       acc = (NI >= 4) ? fma(acc3, ph3[l3], acc) : acc3;
+    }
     }
     c.res = fma(acc, prod, c.res);
     c.b += cnt(R, NI) << J;
@@ -282,6 +379,7 @@ struct Trie {
 
   template <int J, int R>
   static __device__ __forceinline__ void split4(Ctx& c, uint32_t P, T prod) {
+    static_assert(!HREG, "split blocks read the dimension-3 hat table");
     for (int l3 = 0; l3 < R - kTail3; ++l3) {
       const T ph = c.phs[(1 * NM + l3) * NT];
       const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
@@ -354,11 +452,12 @@ struct Trie {
 // One launch evaluates the level groups J0..J1 (compile time) for every
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
+          int CHUNK = 0>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -389,7 +488,10 @@ __global__ void __launch_bounds__(NT, MINB)
         uint32_t cell;
         const T h = hat_cell<T>(xt, l, cell);
         if (t < 2) c.ph[t < 2 ? t : 0][l] = h;
-        else if (t < I) sm[((t - 2) * NM + l) * NT + tid] = h;
+        else if (t < I) {
+          if constexpr (HREG) c.xin[t - 2 < 2 ? t - 2 : 0] = xt;
+          else sm[((t - 2) * NM + l) * NT + tid] = h;
+        }
         else sm[(TR::SM_IN + l) * NT + tid] = h;
       }
     } else {
@@ -407,12 +509,13 @@ __global__ void __launch_bounds__(NT, MINB)
   }
 }
 
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
+          int CHUNK = 0>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK>;
   const size_t smem = TR::smem_bytes;
   static bool attr_set = false;
   if (!attr_set) {
