@@ -26,7 +26,8 @@ timeout 420 ncu --set full --clock-control none --import-source on -k regex:k_ev
 timeout 120 python scripts/ncu_summary.py /tmp/${TAG}_eval.ncu-rep > gpurun_out/${TAG}_eval_ncu.txt 2>&1
 timeout 120 ncu -i /tmp/${TAG}_eval.ncu-rep --page source --csv --print-source sass > /tmp/${TAG}_src.csv 2>/dev/null
 timeout 120 python scripts/ncu_mix.py /tmp/${TAG}_src.csv > gpurun_out/${TAG}_eval_mix.txt 2>&1
-timeout 300 ncu --set full --clock-control none --import-source on -k regex:k_hier -c 2 -o /tmp/${TAG}_hier \
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:k_hier_family -c 2 -o /tmp/${TAG}_hier \
   python bench.py --steps 1 --warmup 0 --m 100000 --no-e2e --no-cpu > gpurun_out/${TAG}_ncu_hier.log 2>&1
 timeout 120 python scripts/ncu_summary.py /tmp/${TAG}_hier.ncu-rep > gpurun_out/${TAG}_hier_ncu.txt 2>&1
+timeout 600 python scripts/bench_configs.py --reps 5 > gpurun_out/${TAG}_configs.txt 2>&1
 ls -la gpurun_out

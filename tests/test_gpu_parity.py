@@ -118,6 +118,23 @@ def test_hierarchize_bit_exact_fp64(P, torch, oracle, d, n):
     np.testing.assert_array_equal(got, want)
 
 
+def test_hierarchize_table_reuse_and_fp32(P, torch, oracle):
+    """The pole-family tables are built on the first call and reused: a second
+    and third hierarchization on the same handle (other data, other dtype)
+    stay bit-exact / within fp32 rounding of the oracle."""
+    d, n = 4, 7
+    g = P.Grid(d, n)
+    xs = oracle.coords(d, n)
+    for k in range(2):
+        v = S.f_A(xs) * (1.0 + k) + 0.1 * np.cos((3.0 + k) * xs.sum(1))
+        got = g.hierarchize_(torch.from_numpy(v).cuda()).cpu().numpy()
+        np.testing.assert_array_equal(got, oracle.hierarchize(d, n, v))
+    v32 = (S.f_A(xs) - 0.2 * np.sin(2.0 * xs.prod(1))).astype(np.float32)
+    got32 = g.hierarchize_(torch.from_numpy(v32).cuda()).cpu().numpy().astype(np.float64)
+    want = oracle.hierarchize(d, n, v32.astype(np.float64))
+    np.testing.assert_allclose(got32, want, rtol=0, atol=64 * d * np.finfo(np.float32).eps * np.abs(v32).max())
+
+
 @pytest.mark.parametrize("d,n", [(1, 17), (2, 15)])
 def test_hierarchize_large_families_fallback(P, torch, oracle, d, n):
     # 2^n - 1 values per pole family exceed shared memory: global ping-pong kernel
