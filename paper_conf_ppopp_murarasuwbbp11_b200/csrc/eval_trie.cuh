@@ -42,7 +42,7 @@ namespace sg {
 namespace trie {
 
 template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0>
+          int CHUNK = 0, int FULL = 4>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
@@ -251,7 +251,7 @@ struct Trie {
   // FLAT = 0, 6.12e6 vs 6.79e6 evals/s), so FLAT defaults to 0.  SYNC adds a
   // CTA barrier per dimension-(I+1) node (experiment; slower at 384x1).
   static constexpr int kFlat = FLAT;  // straight-line sub-trie size (terms)
-  static constexpr int kFull = 4;    // dimension I: unroll every l_I when B <= kFull
+  static constexpr int kFull = FULL;  // dimension I: unroll every l_I when B <= kFull
   static constexpr int kTail = TAIL;  // dimension I: merge the blocks R <= kTail into one basic block
 
   static constexpr uint32_t binom(int a, int b) {
@@ -453,11 +453,11 @@ struct Trie {
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0>
+          int CHUNK = 0, int FULL = 4>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -510,12 +510,12 @@ __global__ void __launch_bounds__(NT, MINB)
 }
 
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0>
+          int CHUNK = 0, int FULL = 4>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL>;
   const size_t smem = TR::smem_bytes;
   static bool attr_set = false;
   if (!attr_set) {
