@@ -11,6 +11,10 @@ namespace sg {
   sg_status name(const Layout& L, const T* a, const T* x, const uint32_t* p, uint64_t m, T* y, cudaStream_t s);
 SG_DECL(trie_d10n11_a, double)
 SG_DECL(trie_d10n11_b, double)
+SG_DECL(trie_d10n11_a_c384, double)
+SG_DECL(trie_d10n11_b_c384, double)
+SG_DECL(trie_d10n11_a_c192, double)
+SG_DECL(trie_d10n11_b_c192, double)
 SG_DECL(trie_d2n3, double)
 SG_DECL(trie_d5n8, double)
 SG_DECL(trie_d5n10, double)
@@ -30,6 +34,15 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     const double* xx = (const double*)x;
     double* yy = (double*)y;
     if (d == 10 && n == 11) {
+      static const char* var = getenv("SG_TRIE_VAR");  // experiment switch
+      if (var && var[0] == '3') {
+        sg_status st = trie_d10n11_a_c384(L, a, xx, perm, m, yy, s);
+        return st == SG_OK ? trie_d10n11_b_c384(L, a, xx, perm, m, yy, s) : st;
+      }
+      if (var && var[0] == '1') {
+        sg_status st = trie_d10n11_a_c192(L, a, xx, perm, m, yy, s);
+        return st == SG_OK ? trie_d10n11_b_c192(L, a, xx, perm, m, yy, s) : st;
+      }
       sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
       if (st != SG_OK) return st;
       return trie_d10n11_b(L, a, xx, perm, m, yy, s);
