@@ -21,6 +21,10 @@ SG_DECL(trie_d5n10, double)
 SG_DECL(trie_d3n14f, float)
 SG_DECL(trie_d20n6, double)
 #undef SG_DECL
+sg_status trie_d10n11_b_hint(int ch, const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                             double* y, cudaStream_t s);
+sg_status trie_d10n11_h4(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
+                         cudaStream_t s);
 
 sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                            void* y, sg_dtype dt, cudaStream_t s, bool* handled) {
@@ -39,6 +43,12 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
         sg_status st = trie_d10n11_a_c384(L, a, xx, perm, m, yy, s);
         return st == SG_OK ? trie_d10n11_b_c384(L, a, xx, perm, m, yy, s) : st;
       }
+      if (var && (var[0] == 'N' || var[0] == 'F' || var[0] == 'E')) {  // L1 hint on groups 9-10
+        sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
+        const int ch = var[0] == 'N' ? 1 : (var[0] == 'F' ? 2 : 3);
+        return st == SG_OK ? trie_d10n11_b_hint(ch, L, a, xx, perm, m, yy, s) : st;
+      }
+      if (var && var[0] == 'H') return trie_d10n11_h4(L, a, xx, perm, m, yy, s);
       if (var && var[0] == '1') {
         sg_status st = trie_d10n11_a_c192(L, a, xx, perm, m, yy, s);
         return st == SG_OK ? trie_d10n11_b_c192(L, a, xx, perm, m, yy, s) : st;

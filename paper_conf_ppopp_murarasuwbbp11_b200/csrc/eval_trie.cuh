@@ -41,8 +41,23 @@
 namespace sg {
 namespace trie {
 
+// Surplus gather with an L1 cache-eviction hint (CH): 0 = plain ld.global.nc,
+// 1 = L1::no_allocate, 2 = L1::evict_first, 3 = L1::evict_last.
+template <int CH, typename T>
+__device__ __forceinline__ T ld_surplus(const T* p) {
+  if constexpr (CH == 0 || sizeof(T) != 8) {
+    return __ldg(p);
+  } else {
+    double v;
+    if constexpr (CH == 1) asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    else if constexpr (CH == 2) asm("ld.global.nc.L1::evict_first.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    else asm("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    return (T)v;
+  }
+}
+
 template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
@@ -56,8 +71,12 @@ struct Trie {
   // accumulation).  Experiment, off: 15 vs 13 loads in flight at first use
   // in SASS, but no measurable change (6.87e6 vs 6.91e6 evals/s).
   static constexpr int SM_IN = HREG ? 0 : 2 * NM;
-  static constexpr int SM_PH = O > 0 ? NM : 0;
-  static constexpr int SM_X = O > 1 ? O - 1 : 0;
+  // H4: hat values of dimension I by exact doubling along its loop (like the
+  // dimensions > I) instead of an NM-row shared-memory table; x_I is then row
+  // 0 of the x table (less shared memory, more L1 for the gathers)
+  static constexpr int SM_PH = (O > 0 && !H4) ? NM : 0;
+  static constexpr int SM_X = H4 ? O : (O > 1 ? O - 1 : 0);
+  static constexpr int xrow(int t) { return H4 ? t - I : t - I - 1; }
   static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X) * NT * sizeof(T);
 
   struct Ctx {
@@ -220,7 +239,7 @@ struct Trie {
           asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
           const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
           asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
-          const T a = __ldg(p + ((uint32_t)cidx << J));
+          const T a = ld_surplus<CH>(p + ((uint32_t)cidx << J));
           if (NI >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[NI > 1 ? 1 : 0][l1], acc2);
           else acc2 = fma(a, c.ph[0][l0], acc2);
           ++cidx;
@@ -276,13 +295,13 @@ struct Trie {
   // dimension I (the innermost outer dimension) at compile-time budget B:
   // levels l = L .. B unrolled into one basic block
   template <int J, int B, int L>
-  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod) {
+  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod, T u) {
     if constexpr (L <= B) {
       constexpr int SG = J - B;
-      const T ph = c.phs[(SM_IN + L) * NT];
+      const T ph = H4 ? hat_u(u) : c.phs[(SM_IN + L) * NT];
       const uint32_t kt = c.K[I] >> (NM - 1 - L);
       block<J, B - L>(c, P | (kt << SG), prod * ph);
-      inner_unrolled<J, B, L + 1>(c, P, prod);
+      inner_unrolled<J, B, L + 1>(c, P, prod, H4 ? dbl_u(u) : u);
     }
   }
 
@@ -299,8 +318,8 @@ struct Trie {
   template <int J, int t, int B>
   static __device__ __forceinline__ void flat(Ctx& c, uint32_t P, T prod) {
     if constexpr (t < I) block<J, B>(c, P, prod);
-    else if constexpr (t == I) inner_unrolled<J, B, 0>(c, P, prod);
-    else flat_level<J, t, B, 0>(c, P, prod, c.xs[(t - I - 1) * NT]);
+    else if constexpr (t == I) inner_unrolled<J, B, 0>(c, P, prod, H4 ? c.xs[xrow(I) * NT] : T(0));
+    else flat_level<J, t, B, 0>(c, P, prod, c.xs[xrow(t) * NT]);
   }
   template <int t>
   static constexpr int flat_max() {  // largest budget whose sub-trie at t is straight-line
@@ -329,13 +348,13 @@ struct Trie {
   // tail of dimension I at run-time budget B: the blocks R = RT .. 0
   // (l_I = B - R), merged into one basic block
   template <int J, int RT>
-  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod) {
+  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod, T u) {
     if constexpr (RT >= 0) {
       const int lt = B - RT;
-      const T ph = c.phs[(SM_IN + lt) * NT];
+      const T ph = H4 ? hat_u(u) : c.phs[(SM_IN + lt) * NT];
       const uint32_t kt = c.K[I] >> (NM - 1 - lt);
       block<J, RT>(c, P | (kt << (J - B)), prod * ph);
-      inner_tail<J, RT - 1>(c, B, P, prod);
+      inner_tail<J, RT - 1>(c, B, P, prod, H4 ? dbl_u(u) : u);
     }
   }
 
@@ -417,14 +436,16 @@ struct Trie {
     }
     const int SG = J - B;  // shift of dimension t's digit
     if constexpr (t == I) {
+      T u = H4 ? c.xs[xrow(I) * NT] : T(0);  // u at level lt (H4)
       for (int lt = 0; lt < B - kTail; ++lt) {
-        const T ph = c.phs[(SM_IN + lt) * NT];
+        const T ph = H4 ? hat_u(u) : c.phs[(SM_IN + lt) * NT];
         const uint32_t kt = c.K[I] >> (NM - 1 - lt);
         leaf<J>(c, B - lt, P | (kt << SG), prod * ph);
+        if constexpr (H4) u = dbl_u(u);
       }
-      inner_tail<J, kTail>(c, B, P, prod);
+      inner_tail<J, kTail>(c, B, P, prod, u);
     } else {
-      T u = c.xs[(t - I - 1) * NT];
+      T u = c.xs[xrow(t) * NT];
       for (int lt = 0; lt <= B; ++lt) {
         // SYNC: keep the warps of a CTA on the same sub-trie (shared L1 sectors
         // and instruction-cache lines); the enumeration is CTA-uniform
@@ -453,11 +474,11 @@ struct Trie {
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -482,7 +503,7 @@ __global__ void __launch_bounds__(NT, MINB)
     kf = kf > T(0) ? kf : T(0);
     kf = kf < fine - T(1) ? kf : fine - T(1);
     c.K[t] = (uint32_t)kf;
-    if (t <= I) {
+    if (t < I || (t == I && !H4)) {
 #pragma unroll
       for (int l = 0; l < NM; ++l) {
         uint32_t cell;
@@ -495,7 +516,7 @@ __global__ void __launch_bounds__(NT, MINB)
         else sm[(TR::SM_IN + l) * NT + tid] = h;
       }
     } else {
-      sm[(TR::SM_IN + TR::SM_PH + (t - I - 1)) * NT + tid] = xt;
+      sm[(TR::SM_IN + TR::SM_PH + TR::xrow(t)) * NT + tid] = xt;
     }
   }
   // (no barrier: every lane reads only its own shared-memory column)
@@ -510,12 +531,12 @@ __global__ void __launch_bounds__(NT, MINB)
 }
 
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4>;
   const size_t smem = TR::smem_bytes;
   static bool attr_set = false;
   if (!attr_set) {
