@@ -20,6 +20,7 @@ SG_DECL(trie_d5n8, double)
 SG_DECL(trie_d5n10, double)
 SG_DECL(trie_d3n14f, float)
 SG_DECL(trie_d20n6, double)
+SG_DECL(trie_d20n6_nos0, double)
 #undef SG_DECL
 sg_status trie_d10n11_b_hint(int ch, const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
                              double* y, cudaStream_t s);
@@ -60,7 +61,11 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     if (d == 2 && n == 3) return trie_d2n3(L, a, xx, perm, m, yy, s);
     if (d == 5 && n == 8) return trie_d5n8(L, a, xx, perm, m, yy, s);
     if (d == 5 && n == 10) return trie_d5n10(L, a, xx, perm, m, yy, s);
-    if (d == 20 && n == 6) return trie_d20n6(L, a, xx, perm, m, yy, s);
+    if (d == 20 && n == 6) {
+      static const char* var = getenv("SG_TRIE_VAR");  // experiment switch
+      if (var && var[0] == 'Z') return trie_d20n6_nos0(L, a, xx, perm, m, yy, s);
+      return trie_d20n6(L, a, xx, perm, m, yy, s);
+    }
   } else {
     if (d == 3 && n == 14) return trie_d3n14f(L, (const float*)alpha, (const float*)x, perm, m, (float*)y, s);
   }

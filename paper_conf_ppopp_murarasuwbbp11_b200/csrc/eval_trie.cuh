@@ -57,7 +57,7 @@ __device__ __forceinline__ T ld_surplus(const T* p) {
 }
 
 template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
@@ -77,12 +77,18 @@ struct Trie {
   static constexpr int SM_PH = (O > 0 && !H4) ? NM : 0;
   static constexpr int SM_X = H4 ? O : (O > 1 ? O - 1 : 0);
   static constexpr int xrow(int t) { return H4 ? t - I : t - I - 1; }
-  static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X) * NT * sizeof(T);
+  // S0: suffix products P0[t] = prod_{u <= t} phi_0(x_u), t = I..D-1, so that a
+  // sub-trie whose level budget is exhausted (every level of dimensions t..0
+  // is 0: one term, one surplus) costs one gather and one FMA instead of a
+  // chain of t - I + 1 hat evaluations (matters at high d: cfg5, d = 20)
+  static constexpr int SM_S0 = (S0 && O > 0) ? O : 0;
+  static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X + SM_S0) * NT * sizeof(T);
 
   struct Ctx {
     const T* __restrict__ alpha;
     const T* phs;  // this lane's column of the hat tables (dims 2, 3, I)
     const T* xs;   // this lane's column of the x table of dimensions > I
+    const T* s0;   // S0: this lane's column of the level-0 suffix products
     T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
     T xin[2];                 // HREG: x of dimensions 2, 3
     uint32_t K[D];
@@ -317,7 +323,13 @@ struct Trie {
   }
   template <int J, int t, int B>
   static __device__ __forceinline__ void flat(Ctx& c, uint32_t P, T prod) {
-    if constexpr (t < I) block<J, B>(c, P, prod);
+    if constexpr (S0 && B == 0 && t >= I) {
+      // every level of dimensions t..0 is 0: the single subspace of this
+      // sub-trie, cell 0 in each of those dimensions (digits of length 0)
+      const T a = ld_surplus<CH>(c.alpha + c.b + P);
+      c.res = fma(a, prod * c.s0[(t - I) * NT], c.res);
+      c.b += 1u << J;
+    } else if constexpr (t < I) block<J, B>(c, P, prod);
     else if constexpr (t == I) inner_unrolled<J, B, 0>(c, P, prod, H4 ? c.xs[xrow(I) * NT] : T(0));
     else flat_level<J, t, B, 0>(c, P, prod, c.xs[xrow(t) * NT]);
   }
@@ -474,11 +486,11 @@ struct Trie {
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -491,6 +503,8 @@ __global__ void __launch_bounds__(NT, MINB)
   c.alpha = alpha;
   c.phs = sm + tid;
   c.xs = sm + (TR::SM_IN + TR::SM_PH) * NT + tid;
+  c.s0 = sm + (TR::SM_IN + TR::SM_PH + TR::SM_X) * NT + tid;
+  T p0 = T(1);  // S0: running product of the level-0 hat values
   // ---- a2: finest cells of every dimension; hat values of every level of
   // dimensions 0..I (registers for 0, 1; shared memory for 2, 3, I)
   bool bad = false;
@@ -503,6 +517,11 @@ __global__ void __launch_bounds__(NT, MINB)
     kf = kf > T(0) ? kf : T(0);
     kf = kf < fine - T(1) ? kf : fine - T(1);
     c.K[t] = (uint32_t)kf;
+    if constexpr (TR::SM_S0 > 0) {
+      uint32_t cell0;
+      p0 *= hat_cell<T>(xt, 0, cell0);
+      if (t >= I) sm[(TR::SM_IN + TR::SM_PH + TR::SM_X + (t - I)) * NT + tid] = p0;
+    }
     if (t < I || (t == I && !H4)) {
 #pragma unroll
       for (int l = 0; l < NM; ++l) {
@@ -531,12 +550,12 @@ __global__ void __launch_bounds__(NT, MINB)
 }
 
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0>;
   const size_t smem = TR::smem_bytes;
   static bool attr_set = false;
   if (!attr_set) {

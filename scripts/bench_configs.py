@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Device-timed sg_evaluate / sg_hierarchize throughput for every BASELINE.json config (1 GPU).
 
-    python scripts/bench_configs.py [--reps 5] > profiles/rNN_configs.txt
+    python scripts/bench_configs.py [--reps 5] [--only cfg3,cfg5] > profiles/rNN_configs.txt
 
 Per config: evaluations/s of sg_evaluate (Morton ordering + evaluation kernels
 + scatter, CUDA events around the call on the current stream, median of
@@ -44,7 +44,10 @@ def main():
     pk_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     f_mhz = json.load(open(pk_path)).get("sm_max_mhz", 1965.0) if os.path.exists(pk_path) else 1965.0
     torch.cuda.set_device(0)
-    for name in ["cfg1", "cfg2", "cfg2p", "cfg3", "cfg4", "cfg5"]:
+    names = ["cfg1", "cfg2", "cfg2p", "cfg3", "cfg4", "cfg5"]
+    if "--only" in sys.argv:
+        names = sys.argv[sys.argv.index("--only") + 1].split(",")
+    for name in names:
         c = S.CONFIGS[name]
         d, n = c["d"], c["n"]
         dt = torch.float32 if c["dtype"] == "f32" else torch.float64
