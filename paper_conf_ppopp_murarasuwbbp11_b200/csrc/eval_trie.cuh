@@ -438,10 +438,58 @@ struct Trie {
   }
 #undef SG_TRIE_CASE
 
+  // S0, budget 1 at dimension t > I: the t + 1 subspaces with one level-1
+  // dimension u (u = 0..t, in the bijection order, Alg. 3: u = 0 first) and
+  // every other level of dimensions t..0 zero are consecutive; dimension u's
+  // one-bit digit k_u(1) sits just above the outer digits P (bit J - 1).
+  // Horner over u: acc <- acc * phi_0(x_u) + alpha_u * phi_1(x_u) * prod_{v<u} phi_0(x_v),
+  // so that acc = sum_u alpha_u phi_1(x_u) prod_{v<=t, v!=u} phi_0(x_v)
+  // (Alg. 7's product of hat values).
+  template <int J, int t>
+  static __device__ __forceinline__ void budget1(Ctx& c, uint32_t P, T prod) {
+    const T* base = c.alpha + c.b + P;
+    T acc = T(0), pre = T(1);
+#pragma unroll
+    for (int u = 0; u <= I; ++u) {
+      T f0, f1;
+      if (u < 2) {
+        f0 = c.ph[u < 2 ? u : 0][0];
+        f1 = c.ph[u < 2 ? u : 0][1];
+      } else if (u < I) {
+        f0 = c.phs[((u - 2) * NM + 0) * NT];
+        f1 = c.phs[((u - 2) * NM + 1) * NT];
+      } else {
+        f0 = c.phs[(SM_IN + 0) * NT];
+        f1 = c.phs[(SM_IN + 1) * NT];
+      }
+      const uint32_t k1 = (c.K[u] >> (NM - 2)) & 1u;
+      const T a = ld_surplus<CH>(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
+      acc = fma(acc, f0, a * f1 * pre);
+      pre *= f0;
+    }
+#pragma unroll 4
+    for (int u = I + 1; u <= t; ++u) {
+      const T x = c.xs[xrow(u) * NT];
+      const T f0 = hat_u(x), f1 = hat_u(dbl_u(x));
+      const uint32_t k1 = x >= T(0.5) ? 1u : 0u;  // = k_u(1) = bit NM-2 of K_u (clamped cells)
+      const T a = ld_surplus<CH>(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
+      acc = fma(acc, f0, a * f1 * pre);
+      pre *= f0;
+    }
+    c.res = fma(acc, prod, c.res);
+    c.b += (uint32_t)(t + 1) << J;
+  }
+
   // node at dimension t >= I with run-time budget B (levels of dimensions
   // t..0 sum to B): a run-time loop over l_t, each child inlined once
   template <int J, int t>
   static __device__ __forceinline__ void node(Ctx& c, int B, uint32_t P, T prod) {
+    if constexpr (S0 && !H4 && I == 4 && t > I && J >= 1 && NM >= 2) {
+      if (B == 1) {
+        budget1<J, t>(c, P, prod);
+        return;
+      }
+    }
     if (B <= flat_max<t>()) {
       flat_dispatch<J, t>(c, B, P, prod);
       return;

@@ -105,9 +105,10 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
   p += align_up(m * 4);
   size_t temp = cub_temp_bytes(m);
   const int d = g->L.d, bits = morton_bits(d);
-  // lag cap: bits / 2 (SG_MORTON_LAGCAP overrides it -- experiment switch)
+  // lag cap 1: measured best at cfg3 (d = 10, m = 10^7: 7.01-7.05e6 evals/s vs 6.92e6 at caps 2-6 and
+  // 6.94e6 at 0, profiles/r01_v5_variants.txt); SG_MORTON_LAGCAP overrides it (experiment switch)
   static const char* capenv = getenv("SG_MORTON_LAGCAP");
-  const int cap = capenv ? atoi(capenv) : bits / 2;
+  const int cap = capenv ? atoi(capenv) : (bits / 2 < 1 ? bits / 2 : 1);
   uint64_t blocks = (m + kThreads - 1) / kThreads;
   if (blocks > (uint64_t)kNumSMs * 32) blocks = (uint64_t)kNumSMs * 32;
   if (dt == SG_F64)
