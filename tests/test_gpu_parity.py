@@ -329,6 +329,35 @@ def test_evaluate_edge_cases(P, torch, oracle, dt):
     check_eval(yg, yo, ao, TOL[dt], "grid points")
 
 
+@pytest.mark.parametrize("d,n", [(5, 8), (20, 6)])
+def test_evaluate_edge_cases_specialised(P, torch, oracle, d, n):
+    """Edge cases through the specialised trie kernels (cfg2 d=5 n=8; cfg5 d=20
+    n=6 with the level-0 suffix products and the budget-1 Horner pass, whose
+    level-1 digit is taken from x >= 0.5): dyadic coordinates (cell
+    boundaries at every level), 0.5 exactly, 1 - 2^-40, tiny, and rows with
+    one coordinate on / outside the boundary (value 0) or NaN."""
+    g = P.Grid(d, n)
+    alpha = hierarchized_alpha(torch, P, g, "B", "f64", seed=d)
+    rng = np.random.default_rng(100 + d)
+    pool = np.array([0.5, 0.25, 0.75, 1.0 / 64, 63.0 / 64, 2.0 ** -30, 1.0 - 2.0 ** -40, 0.375, 0.625])
+    m = 48
+    x = rng.random((m, d))
+    special = rng.random((m, d)) < 0.6
+    x[special] = rng.choice(pool, size=int(special.sum()))
+    x[0, :] = 0.5
+    bad = {1: 0.0, 2: 1.0, 3: -0.25, 4: 1.5, 5: np.inf}
+    for r, v in bad.items():
+        x[r, rng.integers(d)] = v
+    x[6, d - 1] = np.nan
+    xt = torch.tensor(x, dtype=torch.float64, device="cuda")
+    y = g.evaluate(alpha, xt).cpu().numpy()
+    yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy(), x)
+    assert np.isnan(y[6]) and np.isnan(yo[6])
+    assert np.all(y[list(bad)] == 0.0)
+    ok = ~np.isnan(yo)
+    check_eval(y[ok], yo[ok], ao[ok], TOL["f64"], f"edge d={d}")
+
+
 @pytest.mark.parametrize("m", [1, 31, 33, 1000, 4097])
 def test_evaluate_ragged_sizes(P, torch, oracle, m):
     d, n = 5, 6
