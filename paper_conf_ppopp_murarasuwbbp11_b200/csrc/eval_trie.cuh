@@ -82,13 +82,18 @@ struct Trie {
   // is 0: one term, one surplus) costs one gather and one FMA instead of a
   // chain of t - I + 1 hat evaluations (matters at high d: cfg5, d = 20)
   static constexpr int SM_S0 = (S0 && O > 0) ? O : 0;
-  static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X + SM_S0) * NT * sizeof(T);
+  // S0 (budget-1 sub-tries): rho_u = phi_1(x_u) / phi_0(x_u) in [0, 2] (0 where
+  // phi_0 = 0, i.e. x outside (0,1), where phi_1 = 0 too), with the level-1
+  // cell k_u(1) in its sign bit; one row per dimension
+  static constexpr int SM_RHO = (S0 && O > 0 && NM >= 2) ? D : 0;
+  static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X + SM_S0 + SM_RHO) * NT * sizeof(T);
 
   struct Ctx {
     const T* __restrict__ alpha;
     const T* phs;  // this lane's column of the hat tables (dims 2, 3, I)
     const T* xs;   // this lane's column of the x table of dimensions > I
     const T* s0;   // S0: this lane's column of the level-0 suffix products
+    const T* rho;  // S0: this lane's column of the signed level-1/level-0 hat ratios
     T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
     T xin[2];                 // HREG: x of dimensions 2, 3
     uint32_t K[D];
@@ -447,36 +452,17 @@ struct Trie {
   // (Alg. 7's product of hat values).
   template <int J, int t>
   static __device__ __forceinline__ void budget1(Ctx& c, uint32_t P, T prod) {
+    // sum_u alpha_u phi_1(x_u) prod_{v<=t, v!=u} phi_0(x_v) = S0[t] * sum_u alpha_u rho_u
     const T* base = c.alpha + c.b + P;
-    T acc = T(0), pre = T(1);
+    T acc = T(0);
 #pragma unroll
-    for (int u = 0; u <= I; ++u) {
-      T f0, f1;
-      if (u < 2) {
-        f0 = c.ph[u < 2 ? u : 0][0];
-        f1 = c.ph[u < 2 ? u : 0][1];
-      } else if (u < I) {
-        f0 = c.phs[((u - 2) * NM + 0) * NT];
-        f1 = c.phs[((u - 2) * NM + 1) * NT];
-      } else {
-        f0 = c.phs[(SM_IN + 0) * NT];
-        f1 = c.phs[(SM_IN + 1) * NT];
-      }
-      const uint32_t k1 = (c.K[u] >> (NM - 2)) & 1u;
+    for (int u = 0; u <= t; ++u) {
+      const T r = c.rho[u * NT];
+      const uint32_t k1 = (uint32_t)__double2hiint((double)r) >> 31;  // k_u(1), the sign bit
       const T a = ld_surplus<CH>(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
-      acc = fma(acc, f0, a * f1 * pre);
-      pre *= f0;
+      acc = fma(a, fabs(r), acc);
     }
-#pragma unroll 4
-    for (int u = I + 1; u <= t; ++u) {
-      const T x = c.xs[xrow(u) * NT];
-      const T f0 = hat_u(x), f1 = hat_u(dbl_u(x));
-      const uint32_t k1 = x >= T(0.5) ? 1u : 0u;  // = k_u(1) = bit NM-2 of K_u (clamped cells)
-      const T a = ld_surplus<CH>(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
-      acc = fma(acc, f0, a * f1 * pre);
-      pre *= f0;
-    }
-    c.res = fma(acc, prod, c.res);
+    c.res = fma(acc, prod * c.s0[(t - I) * NT], c.res);
     c.b += (uint32_t)(t + 1) << J;
   }
 
@@ -552,6 +538,7 @@ __global__ void __launch_bounds__(NT, MINB)
   c.phs = sm + tid;
   c.xs = sm + (TR::SM_IN + TR::SM_PH) * NT + tid;
   c.s0 = sm + (TR::SM_IN + TR::SM_PH + TR::SM_X) * NT + tid;
+  c.rho = sm + (TR::SM_IN + TR::SM_PH + TR::SM_X + TR::SM_S0) * NT + tid;
   T p0 = T(1);  // S0: running product of the level-0 hat values
   // ---- a2: finest cells of every dimension; hat values of every level of
   // dimensions 0..I (registers for 0, 1; shared memory for 2, 3, I)
@@ -569,6 +556,13 @@ __global__ void __launch_bounds__(NT, MINB)
       uint32_t cell0;
       p0 *= hat_cell<T>(xt, 0, cell0);
       if (t >= I) sm[(TR::SM_IN + TR::SM_PH + TR::SM_X + (t - I)) * NT + tid] = p0;
+    }
+    if constexpr (TR::SM_RHO > 0) {
+      uint32_t c0, c1;
+      const T f0 = hat_cell<T>(xt, 0, c0), f1 = hat_cell<T>(xt, 1, c1);
+      const double r = f0 > T(0) ? (double)(f1 / f0) : 0.0;
+      const long long bits = __double_as_longlong(r) | ((long long)(c1 & 1u) << 63);
+      sm[(TR::SM_IN + TR::SM_PH + TR::SM_X + TR::SM_S0 + t) * NT + tid] = (T)__longlong_as_double(bits);
     }
     if (t < I || (t == I && !H4)) {
 #pragma unroll

@@ -7,7 +7,7 @@ timeout 300 python scripts/bench_configs.py --reps 5 --only cfg5 > gpurun_out/${
 SG_TRIE_VAR=Z timeout 300 python scripts/bench_configs.py --reps 5 --only cfg5 > gpurun_out/${T}_cfg_off.txt 2>&1
 timeout 300 python -m pytest tests -m gpu -x -q > gpurun_out/${T}_pytest_all.log 2>&1; echo "pytest exit $?" >> gpurun_out/${T}_pytest_all.log
 i=0
-for E in "" SG_MORTON_LAGCAP=1 SG_MORTON_LAGCAP=0 "" SG_MORTON_LAGCAP=1 SG_MORTON_LAGCAP=0; do
+for E in ${LAGS:-}; do
   env $E timeout 240 python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu > gpurun_out/${T}_lag$i.log 2>&1
   echo "env=[$E] exit $?" >> gpurun_out/${T}_lag$i.log
   i=$((i+1))
