@@ -123,3 +123,26 @@ def test_device_calls_without_gpu_fail_loudly(P):
         assert _sg.lib.sg_hierarchize(h, ctypes.c_void_p(8), 0, None) == _sg.SG_ERR_NODEV
     finally:
         P.sg_destroy(h)
+
+
+def test_budget1_hat_ratio_reading():
+    """DESIGN.md 6.1 (cfg5 budget-1 sub-tries): the d = 20 kernel sums a
+    budget-1 sub-trie as S0[t] * sum_u alpha_u rho_u with rho = phi_1 / phi_0,
+    which relies on (i) 0 <= phi_1(x) <= 2 phi_0(x) on [0, 1] (bounded,
+    well-conditioned quotient) and (ii) phi_1 = 0 wherever phi_0 = 0.  Hat
+    functions from P:L87, phi_{l,i}(x) = max(0, 1 - |2^{l+1} x - i|), level l
+    having the odd indices i = 1, 3, .., 2^{l+1} - 1 (0-based levels)."""
+    def phi(l, x):  # the one non-zero hat of level l at x (max over the level's cells)
+        i = np.arange(1, 2 ** (l + 1), 2)[None, :]
+        return np.max(np.maximum(0.0, 1.0 - np.abs(2.0 ** (l + 1) * x[:, None] - i)), axis=1)
+
+    x = np.concatenate([np.linspace(-0.5, 1.5, 200001), np.arange(0, 65) / 64.0, [2.0 ** -40, 1 - 2.0 ** -40]])
+    f0, f1 = phi(0, x), phi(1, x)
+    assert np.all(f1 <= 2.0 * f0 + 1e-15)
+    assert np.all(f1[f0 == 0.0] == 0.0)
+    inside = (x > 0) & (x <= 0.25)
+    np.testing.assert_allclose(f1[inside] / f0[inside], 2.0, rtol=1e-12)
+    # the level-1 cell the kernel stores in the sign bit: k(1) = 1 iff x >= 1/2
+    for xv in [0.25, 0.49999999, 0.5, 0.75, 1.0 - 2.0 ** -40]:
+        k = int(np.clip(np.floor(2.0 * xv), 0, 1))
+        assert k == (1 if xv >= 0.5 else 0)
