@@ -36,14 +36,13 @@ inline int morton_bits(int d) {
 // in the curve makes warps compact in dimensions 0..d/2 and elongated in the
 // fast ones: at d = 10 this cuts the modelled L1 cycles per gather from 4.11
 // to 3.27 (SURVEY-style simulation over 10^7 uniform points, groups 5-10).
-__host__ __device__ inline int morton_lag(int t, int d, int bits, int cap) {
-  if (d < 4) return 0;
-  const int lag = t - d / 2;
+__host__ __device__ inline int morton_lag(int t, int start, int cap) {
+  const int lag = t - start;  // start = d / 2 (d >= 4), d (no lag) below
   return lag <= 0 ? 0 : (lag < cap ? lag : cap);
 }
 
 template <typename T>
-__global__ void __launch_bounds__(kThreads) k_morton(const T* __restrict__ x, uint64_t m, int d, int bits, int cap,
+__global__ void __launch_bounds__(kThreads) k_morton(const T* __restrict__ x, uint64_t m, int d, int bits, int cap, int start,
                                                      uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
   for (uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; q < m; q += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t c[SG_MAX_D];
@@ -58,10 +57,10 @@ __global__ void __launch_bounds__(kThreads) k_morton(const T* __restrict__ x, ui
     // bit planes from the most significant one; dimension t enters lag(t)
     // planes late (see morton_lag), so every dimension keeps `bits` bits
     uint64_t key = 0;
-    const int lmax = morton_lag(d - 1, d, bits, cap);
+    const int lmax = morton_lag(d - 1, start, cap);
     for (int p = 0; p < bits + lmax; ++p)
       for (int t = 0; t < d; ++t) {
-        const int b = p - morton_lag(t, d, bits, cap);  // bit of dimension t, 0 = its MSB
+        const int b = p - morton_lag(t, start, cap);  // bit of dimension t, 0 = its MSB
         if (b >= 0 && b < bits) key = (key << 1) | ((c[t] >> (bits - 1 - b)) & 1u);
       }
     keys[q] = key;
@@ -109,12 +108,17 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
   // 6.94e6 at 0, profiles/r01_v5_variants.txt); SG_MORTON_LAGCAP overrides it (experiment switch)
   static const char* capenv = getenv("SG_MORTON_LAGCAP");
   const int cap = capenv ? atoi(capenv) : (bits / 2 < 1 ? bits / 2 : 1);
+  // lag(t) = min(cap, t - start) for t > start; start = d / 2 + 1: measured best at cfg3 (d = 10: dimensions
+  // 7-9 one plane late, 7.08e6 evals/s vs 6.88 / 6.97 / 6.99-7.01 / 7.01e6 at start 3 / 4 / 5 / 7,
+  // profiles/r01_v5_variants.txt); SG_MORTON_LAGSTART overrides it (experiment switch)
+  static const char* startenv = getenv("SG_MORTON_LAGSTART");
+  const int start = d < 4 ? d : (startenv ? atoi(startenv) : d / 2 + 1);
   uint64_t blocks = (m + kThreads - 1) / kThreads;
   if (blocks > (uint64_t)kNumSMs * 32) blocks = (uint64_t)kNumSMs * 32;
   if (dt == SG_F64)
-    k_morton<double><<<(unsigned)blocks, kThreads, 0, s>>>((const double*)x, m, d, bits, cap, k0, v0);
+    k_morton<double><<<(unsigned)blocks, kThreads, 0, s>>>((const double*)x, m, d, bits, cap, start, k0, v0);
   else
-    k_morton<float><<<(unsigned)blocks, kThreads, 0, s>>>((const float*)x, m, d, bits, cap, k0, v0);
+    k_morton<float><<<(unsigned)blocks, kThreads, 0, s>>>((const float*)x, m, d, bits, cap, start, k0, v0);
   sg_status st = launched("k_morton");
   if (st != SG_OK) return st;
   cudaError_t e = cub::DeviceRadixSort::SortPairs(p, temp, k0, k1, v0, v1, (int)m, 0, d * bits, s);
