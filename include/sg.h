@@ -143,11 +143,40 @@ sg_status sg_evaluate_workspace_bytes(sg_grid g, uint64_t m, sg_dtype dt, uint32
 sg_status sg_evaluate(sg_grid g, const void *d_alpha, const void *d_x, uint64_t m, void *d_y, sg_dtype dt,
                       uint32_t flags, void *d_workspace, size_t ws_bytes, void *stream);
 
+/* Row a1 on its own: the space-filling-curve order of a query batch.
+ * d_perm (m uint32, device, caller-owned) receives the permutation that
+ * sorts d_x (m x d, dtype dt) along the Morton curve sg_evaluate uses (the
+ * paper's blocking over evaluation points; coalesced coordinate
+ * staging).  The sort is a stable radix sort of (key, index) pairs,
+ * so the result is a deterministic function of the batch: every process that
+ * orders the same batch obtains the same permutation (multi-GPU ranks agree
+ * on one global order without communicating).  d_workspace must
+ * hold sg_evaluate_workspace_bytes(g, m, dt, 0) bytes, or be NULL (allocated
+ * stream-ordered).  Asynchronous on `stream`. */
+sg_status sg_sfc_order(sg_grid g, const void *d_x, uint64_t m, sg_dtype dt, uint32_t *d_perm, void *d_workspace,
+                       size_t ws_bytes, void *stream);
+
+/* Evaluate one contiguous range of an ordered batch (the multi-GPU shard of
+ * the "embarrassingly parallel" evaluation, Sec. 4.3, with a static
+ * workload distribution):
+ *   for k < count:  q = d_perm[first + k];  d_y[q] = f_s(d_x[q,:]).
+ * d_x (m x d) and d_y (m) are the WHOLE batch in input order (only the
+ * range's rows of d_x are read and only its entries of d_y written);
+ * d_perm (m entries) is an order from sg_sfc_order.  With d_perm == NULL the
+ * batch is taken as already ordered: rows first..first+count-1.  The result
+ * of every query is bitwise independent of the range it is evaluated in.
+ * first + count must be <= m (SG_ERR_RANGE otherwise).  Asynchronous. */
+sg_status sg_evaluate_ordered(sg_grid g, const void *d_alpha, const void *d_x, uint64_t m, const uint32_t *d_perm,
+                              uint64_t first, uint64_t count, void *d_y, sg_dtype dt, void *stream);
+
 /* End-to-end evaluation from HOST buffers: copies h_x (m x d) to the device,
  * evaluates as sg_evaluate, copies the m results to h_y.  d_alpha is on the
- * device.  Device buffers are allocated stream-ordered; the copies are
- * chunked and overlapped with the evaluation.  Returns after the results
- * are in h_y (synchronizes `stream`). */
+ * device.  Device buffers are allocated stream-ordered.  The three steps run
+ * back to back on `stream` (H2D of the whole batch, evaluation, D2H): the
+ * space-filling-curve order needs every query on the device before the
+ * first evaluation launch, and chunking the batch would shrink the warps'
+ * spatial locality.  Returns after the results are in
+ * h_y (synchronizes `stream`). */
 sg_status sg_evaluate_host(sg_grid g, const void *d_alpha, const void *h_x, uint64_t m, void *h_y, sg_dtype dt,
                            uint32_t flags, void *stream);
 

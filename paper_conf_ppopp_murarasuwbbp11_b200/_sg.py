@@ -16,7 +16,8 @@ import numpy as np
 import torch  # loads the CUDA runtime libsg links against
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsg.so")
+# SG_LIB selects another build of the same sources (scripts/gpu_exp.sh: libsg_exp.so); default: the product
+LIB_PATH = os.environ.get("SG_LIB") or os.path.join(_HERE, "libsg.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is not built: run `python paper_conf_ppopp_murarasuwbbp11_b200/build.py` "
@@ -52,6 +53,8 @@ _SIGS = {
     "sg_evaluate_workspace_bytes": [_p, _u64, ctypes.c_int, _u32, ctypes.POINTER(_sz)],
     "sg_evaluate": [_p, _p, _p, _u64, _p, ctypes.c_int, _u32, _p, _sz, _p],
     "sg_evaluate_host": [_p, _p, _p, _u64, _p, ctypes.c_int, _u32, _p],
+    "sg_sfc_order": [_p, _p, _u64, ctypes.c_int, _p, _p, _sz, _p],
+    "sg_evaluate_ordered": [_p, _p, _p, _u64, _p, _u64, _u64, _p, ctypes.c_int, _p],
 }
 for _name, _args in _SIGS.items():
     _f = getattr(lib, _name)
@@ -175,16 +178,56 @@ def sg_evaluate_workspace_bytes(g, m: int, dtype, flags: int = 0) -> int:
     return int(b.value)
 
 
+def _check_batch(alpha: torch.Tensor, x: torch.Tensor, y: torch.Tensor | None = None, num_points: int | None = None,
+                 d: int | None = None):
+    """Shapes / dtypes / devices of one evaluation call (the C ABI takes raw pointers)."""
+    if x.dim() != 2 or (d is not None and x.shape[1] != d):
+        raise ValueError(f"x must be (m, {d if d is not None else 'd'}), got {tuple(x.shape)}")
+    if alpha.dtype != x.dtype:
+        raise ValueError(f"alpha ({alpha.dtype}) and x ({x.dtype}) must have the same dtype")
+    if num_points is not None and alpha.numel() != num_points:
+        raise ValueError(f"alpha has {alpha.numel()} entries, the grid {num_points} points")
+    if y is not None:
+        if y.dtype != x.dtype or y.numel() != x.shape[0] or not y.is_contiguous():
+            raise ValueError(f"out must be a contiguous {x.dtype} tensor of {x.shape[0]} entries")
+        if y.is_cuda != x.is_cuda or (y.is_cuda and y.device != x.device):
+            raise ValueError("out must be on the same device as x")
+
+
 def sg_evaluate(g, alpha: torch.Tensor, x: torch.Tensor, y: torch.Tensor, flags: int = 0,
                 workspace: torch.Tensor | None = None, stream=None) -> None:
+    _check_batch(alpha, x, y)
     ws = _dev(workspace, "workspace") if workspace is not None else None
     wsb = workspace.numel() * workspace.element_size() if workspace is not None else 0
     _check(lib.sg_evaluate(g, _dev(alpha, "alpha"), _dev(x, "x"), x.shape[0], _dev(y, "y"), _dtype_code(x), flags,
                            ws, wsb, _stream(stream)), "sg_evaluate")
 
 
+def sg_sfc_order(g, x: torch.Tensor, perm: torch.Tensor, workspace: torch.Tensor | None = None, stream=None) -> None:
+    """perm (m int32/uint32, device) <- the Morton order of the batch x (deterministic)."""
+    if perm.dtype not in (torch.int32, torch.uint32) or perm.numel() != x.shape[0]:
+        raise ValueError("perm must hold m int32 entries")
+    ws = _dev(workspace, "workspace") if workspace is not None else None
+    wsb = workspace.numel() * workspace.element_size() if workspace is not None else 0
+    _check(lib.sg_sfc_order(g, _dev(x, "x"), x.shape[0], _dtype_code(x), _dev(perm, "perm"), ws, wsb,
+                            _stream(stream)), "sg_sfc_order")
+
+
+def sg_evaluate_ordered(g, alpha: torch.Tensor, x: torch.Tensor, perm: torch.Tensor | None, first: int, count: int,
+                        y: torch.Tensor, stream=None) -> None:
+    """y[perm[first+k]] = f_s(x[perm[first+k]]) for k < count (whole-batch x and y, input order)."""
+    _check_batch(alpha, x, y)
+    if perm is not None and (perm.dtype not in (torch.int32, torch.uint32) or perm.numel() != x.shape[0]):
+        raise ValueError("perm must hold m int32 entries")
+    pp = _dev(perm, "perm") if perm is not None else None
+    _check(lib.sg_evaluate_ordered(g, _dev(alpha, "alpha"), _dev(x, "x"), x.shape[0], pp, first, count, _dev(y, "y"),
+                                   _dtype_code(x), _stream(stream)), "sg_evaluate_ordered")
+
+
 def sg_evaluate_host(g, alpha: torch.Tensor, x_host, y_host, flags: int = 0, stream=None) -> None:
     """x_host / y_host: CPU tensors (pinned for full copy bandwidth) or numpy arrays."""
+    if x_host.shape[0] != y_host.shape[0] or x_host.dtype != y_host.dtype or x_host.dtype != alpha.dtype:
+        raise ValueError("x_host (m, d) and y_host (m) must match alpha's dtype and each other's length")
     xp = x_host.data_ptr() if isinstance(x_host, torch.Tensor) else x_host.ctypes.data
     yp = y_host.data_ptr() if isinstance(y_host, torch.Tensor) else y_host.ctypes.data
     _check(lib.sg_evaluate_host(g, _dev(alpha, "alpha"), xp, x_host.shape[0], yp, _dtype_code(x_host), flags,

@@ -4,6 +4,7 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <mutex>
 
 #include "layout.cuh"
 
@@ -14,8 +15,11 @@ struct sg_grid_s {
   // pole-family tables of the hierarchization (built on first use, per device
   // copy of the grid; hier_kernels.cu): per dimension, per family a packed
   // (|l_{-t}|, suffix sum) word and the offset of its first block base, and
-  // per family per block the global offset of the block
-  void* d_hier_tab = nullptr;
+  // per family per block the global offset of the block.  Built once, under
+  // hier_mu and completed (stream-synchronised) before the pointer is
+  // published, so concurrent callers on any stream see finished tables.
+  mutable std::atomic<void*> d_hier_tab{nullptr};
+  mutable std::mutex hier_mu;
 };
 
 namespace sg {
@@ -34,6 +38,25 @@ inline sg_status launched(const char* what) {
 }
 
 constexpr int kNumSMs = 148;
+
+// Function attributes are per device: opt a kernel into `smem` bytes of dynamic
+// shared memory (and an L1/shared carveout, percent; < 0 = leave it) once per
+// device, tracked in the caller's per-kernel bitmask (devices 0..63).
+template <typename K>
+inline sg_status set_smem_attr(K kern, std::atomic<uint64_t>& done, size_t smem, int carveout, const char* what) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, what);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (done.load(std::memory_order_acquire) & bit) return SG_OK;
+  e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)(smem > 48 * 1024 ? smem : 48 * 1024));
+  if (e == cudaSuccess && carveout >= 0)
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carveout > 100 ? 100 : carveout);
+  if (e != cudaSuccess) return cuda_fail(e, what);
+  done.fetch_or(bit, std::memory_order_release);
+  return SG_OK;
+}
 
 // ---- kernel timing instrumentation (sg_profile_enable / sg_profile_read) ----
 enum ProfKind { kProfEval = 0, kProfHier = 1 };
@@ -54,7 +77,7 @@ sg_status launch_coords(const sg_grid_s* g, uint64_t first, uint64_t count, void
 sg_status launch_hierarchize(const sg_grid_s* g, void* v, sg_dtype dt, cudaStream_t s);
 size_t sfc_workspace_bytes(uint64_t m);
 sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dtype dt, void* ws, size_t ws_bytes,
-                           const uint32_t** perm_out, cudaStream_t s);
+                           uint32_t* perm_dst, const uint32_t** perm_out, cudaStream_t s);
 sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                           void* y, sg_dtype dt, uint32_t flags, cudaStream_t s);
 

@@ -169,13 +169,9 @@ template <typename T, int D, int NM>
 sg_status launch_t(const T* alpha, const T* x, const uint32_t* perm, uint64_t m, int n, T* y, cudaStream_t s) {
   static_assert(D >= 3, "fast kernel needs D >= 3");
   const size_t smem = (size_t)(D - 3) * NM * kThreads * sizeof(T);
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_eval_fast<T, D, NM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(smem > 48 * 1024 ? smem : 48 * 1024));
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_eval_fast)");
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  sg_status st = set_smem_attr(k_eval_fast<T, D, NM>, attr_done, smem, -1, "cudaFuncSetAttribute(k_eval_fast)");
+  if (st != SG_OK) return st;
   const unsigned blocks = (unsigned)((m + kThreads - 1) / kThreads);
   k_eval_fast<T, D, NM><<<blocks, kThreads, smem, s>>>(alpha, x, perm, (uint32_t)m, n, y);
   return launched("k_eval_fast");

@@ -1,8 +1,6 @@
 // eval_trie.cu -- dispatch of the v2 evaluation kernel (eval_trie.cuh) by
 // (d, n, dtype); shapes without an instantiation return handled = false and
 // fall through to eval_fast.cu / eval_simple.cu.
-#include <stdlib.h>
-
 #include "common.cuh"
 
 namespace sg {
@@ -11,21 +9,16 @@ namespace sg {
   sg_status name(const Layout& L, const T* a, const T* x, const uint32_t* p, uint64_t m, T* y, cudaStream_t s);
 SG_DECL(trie_d10n11_a, double)
 SG_DECL(trie_d10n11_b, double)
-SG_DECL(trie_d10n11_a_c384, double)
-SG_DECL(trie_d10n11_b_c384, double)
-SG_DECL(trie_d10n11_a_c192, double)
-SG_DECL(trie_d10n11_b_c192, double)
 SG_DECL(trie_d2n3, double)
 SG_DECL(trie_d5n8, double)
 SG_DECL(trie_d5n10, double)
 SG_DECL(trie_d3n14f, float)
 SG_DECL(trie_d20n6, double)
-SG_DECL(trie_d20n6_nos0, double)
 #undef SG_DECL
-sg_status trie_d10n11_b_hint(int ch, const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
-                             double* y, cudaStream_t s);
-sg_status trie_d10n11_h4(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
-                         cudaStream_t s);
+#ifdef SG_EXP
+bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
+                  sg_dtype dt, cudaStream_t s, sg_status* st);
+#endif
 
 sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                            void* y, sg_dtype dt, cudaStream_t s, bool* handled) {
@@ -34,26 +27,17 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
   const Layout& L = g->L;
   const int d = L.d, n = L.n;
   *handled = true;
+#ifdef SG_EXP
+  {
+    sg_status st = SG_OK;
+    if (exp_dispatch(L, alpha, x, perm, m, y, dt, s, &st)) return st;
+  }
+#endif
   if (dt == SG_F64) {
     const double* a = (const double*)alpha;
     const double* xx = (const double*)x;
     double* yy = (double*)y;
     if (d == 10 && n == 11) {
-      static const char* var = getenv("SG_TRIE_VAR");  // experiment switch
-      if (var && var[0] == '3') {
-        sg_status st = trie_d10n11_a_c384(L, a, xx, perm, m, yy, s);
-        return st == SG_OK ? trie_d10n11_b_c384(L, a, xx, perm, m, yy, s) : st;
-      }
-      if (var && (var[0] == 'N' || var[0] == 'F' || var[0] == 'E')) {  // L1 hint on groups 9-10
-        sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
-        const int ch = var[0] == 'N' ? 1 : (var[0] == 'F' ? 2 : 3);
-        return st == SG_OK ? trie_d10n11_b_hint(ch, L, a, xx, perm, m, yy, s) : st;
-      }
-      if (var && var[0] == 'H') return trie_d10n11_h4(L, a, xx, perm, m, yy, s);
-      if (var && var[0] == '1') {
-        sg_status st = trie_d10n11_a_c192(L, a, xx, perm, m, yy, s);
-        return st == SG_OK ? trie_d10n11_b_c192(L, a, xx, perm, m, yy, s) : st;
-      }
       sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
       if (st != SG_OK) return st;
       return trie_d10n11_b(L, a, xx, perm, m, yy, s);
@@ -62,8 +46,6 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     if (d == 5 && n == 8) return trie_d5n8(L, a, xx, perm, m, yy, s);
     if (d == 5 && n == 10) return trie_d5n10(L, a, xx, perm, m, yy, s);
     if (d == 20 && n == 6) {
-      static const char* var = getenv("SG_TRIE_VAR");  // experiment switch
-      if (var && var[0] == 'Z') return trie_d20n6_nos0(L, a, xx, perm, m, yy, s);
       return trie_d20n6(L, a, xx, perm, m, yy, s);
     }
   } else {

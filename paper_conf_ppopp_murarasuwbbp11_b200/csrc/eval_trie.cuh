@@ -57,8 +57,11 @@ __device__ __forceinline__ T ld_surplus(const T* p) {
 }
 
 template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false, bool GO = false>
 struct Trie {
+  // GO (experiment builds only, SG_EXP): "gather only" -- every hat value is 1, no hat tables are read;
+  // the same surplus gathers, addresses and Horner adds, to measure the memory ceiling of the access stream
+  static __device__ __forceinline__ T phs_at(const T* phs, int row) { return GO ? T(1) : phs[row * NT]; }
   static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
   // shared memory, [row][lane]: hat values of dimensions 2, 3 (loaded per
@@ -214,8 +217,8 @@ struct Trie {
     } else {
 #pragma unroll
       for (int l = 0; l <= R; ++l) {
-        ph2[l] = (NI >= 3) ? c.phs[(0 * NM + l) * NT] : T(1);
-        ph3[l] = (NI >= 4) ? c.phs[(1 * NM + l) * NT] : T(1);
+        ph2[l] = (NI >= 3) ? phs_at(c.phs, 0 * NM + l) : T(1);
+        ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
       }
     }
     T acc = T(0);
@@ -292,6 +295,7 @@ struct Trie {
 
   // hat value from u = 2^l x - k(l) (reading G7): max(0, 2 min(u, 1-u))
   static __device__ __forceinline__ T hat_u(T u) {
+    if constexpr (GO) return T(1);
     const T w = T(1) - u;
     const T mn = u < w ? u : w;
     const T h = mn + mn;
@@ -309,7 +313,7 @@ struct Trie {
   static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod, T u) {
     if constexpr (L <= B) {
       constexpr int SG = J - B;
-      const T ph = H4 ? hat_u(u) : c.phs[(SM_IN + L) * NT];
+      const T ph = H4 ? hat_u(u) : phs_at(c.phs, SM_IN + L);
       const uint32_t kt = c.K[I] >> (NM - 1 - L);
       block<J, B - L>(c, P | (kt << SG), prod * ph);
       inner_unrolled<J, B, L + 1>(c, P, prod, H4 ? dbl_u(u) : u);
@@ -368,7 +372,7 @@ struct Trie {
   static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod, T u) {
     if constexpr (RT >= 0) {
       const int lt = B - RT;
-      const T ph = H4 ? hat_u(u) : c.phs[(SM_IN + lt) * NT];
+      const T ph = H4 ? hat_u(u) : phs_at(c.phs, SM_IN + lt);
       const uint32_t kt = c.K[I] >> (NM - 1 - lt);
       block<J, RT>(c, P | (kt << (J - B)), prod * ph);
       inner_tail<J, RT - 1>(c, B, P, prod, H4 ? dbl_u(u) : u);
@@ -406,7 +410,7 @@ struct Trie {
   static __device__ __forceinline__ void tail3(Ctx& c, uint32_t P, T prod) {
     if constexpr (RT >= 0) {
       constexpr int l3 = R - RT;
-      const T ph = c.phs[(1 * NM + l3) * NT];
+      const T ph = phs_at(c.phs, 1 * NM + l3);
       const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
       block<J, RT, 3>(c, P | (k3 << (J - R)), prod * ph);
       tail3<J, R, RT - 1>(c, P, prod);
@@ -417,7 +421,7 @@ struct Trie {
   static __device__ __forceinline__ void split4(Ctx& c, uint32_t P, T prod) {
     static_assert(!HREG, "split blocks read the dimension-3 hat table");
     for (int l3 = 0; l3 < R - kTail3; ++l3) {
-      const T ph = c.phs[(1 * NM + l3) * NT];
+      const T ph = phs_at(c.phs, 1 * NM + l3);
       const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
       leaf3<J>(c, R - l3, P | (k3 << (J - R)), prod * ph);
     }
@@ -484,7 +488,7 @@ struct Trie {
     if constexpr (t == I) {
       T u = H4 ? c.xs[xrow(I) * NT] : T(0);  // u at level lt (H4)
       for (int lt = 0; lt < B - kTail; ++lt) {
-        const T ph = H4 ? hat_u(u) : c.phs[(SM_IN + lt) * NT];
+        const T ph = H4 ? hat_u(u) : phs_at(c.phs, SM_IN + lt);
         const uint32_t kt = c.K[I] >> (NM - 1 - lt);
         leaf<J>(c, B - lt, P | (kt << SG), prod * ph);
         if constexpr (H4) u = dbl_u(u);
@@ -520,11 +524,11 @@ struct Trie {
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false, bool GO = false>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0, GO>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -568,7 +572,7 @@ __global__ void __launch_bounds__(NT, MINB)
 #pragma unroll
       for (int l = 0; l < NM; ++l) {
         uint32_t cell;
-        const T h = hat_cell<T>(xt, l, cell);
+        const T h = GO ? T(1) : hat_cell<T>(xt, l, cell);
         if (t < 2) c.ph[t < 2 ? t : 0][l] = h;
         else if (t < I) {
           if constexpr (HREG) c.xin[t - 2 < 2 ? t - 2 : 0] = xt;
@@ -592,25 +596,19 @@ __global__ void __launch_bounds__(NT, MINB)
 }
 
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false>
+          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false, bool GO = false>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0>;
+  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0, GO>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0, GO>;
   const size_t smem = TR::smem_bytes;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(smem > 48 * 1024 ? smem : 48 * 1024));
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_eval_trie)");
-    // shared memory only for the per-lane tables: the rest of the 256 KB stays L1
-    // for the surplus gathers
-    const int pct = (int)((smem * MINB * 100 + 227 * 1024 - 1) / (227 * 1024)) + 1;
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, pct > 100 ? 100 : pct);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(carveout)");
-    attr_set = true;
-  }
+  // shared memory only for the per-lane tables: the rest of the 256 KB stays L1
+  // for the surplus gathers
+  const int pct = (int)((smem * MINB * 100 + 227 * 1024 - 1) / (227 * 1024)) + 1;
+  static std::atomic<uint64_t> attr_done{0};
+  const sg_status st = set_smem_attr(kern, attr_done, smem, pct, "cudaFuncSetAttribute(k_eval_trie)");
+  if (st != SG_OK) return st;
   const unsigned blocks = (unsigned)((m + NT - 1) / NT);
   kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, L.n, (uint32_t)L.off[J0], J0 > 0 ? 1 : 0, y);
   return launched("k_eval_trie");

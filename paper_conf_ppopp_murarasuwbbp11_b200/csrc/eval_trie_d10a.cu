@@ -14,20 +14,4 @@ sg_status trie_d10n11_a(const Layout& L, const double* a, const double* x, const
 }
 
 
-sg_status trie_d10n11_a_c384(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
-  sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 384, 1, 0, 6>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 384, 1, 7, 7>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 384, 1, 8, 8>(L, a, x, p, m, y, s);
-  return st;
-}
-
-sg_status trie_d10n11_a_c192(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
-  sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 192, 2, 0, 6>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 192, 2, 7, 7>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 192, 2, 8, 8>(L, a, x, p, m, y, s);
-  return st;
-}
-
 }  // namespace sg

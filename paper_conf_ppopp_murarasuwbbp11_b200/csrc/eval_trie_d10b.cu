@@ -13,18 +13,4 @@ sg_status trie_d10n11_b(const Layout& L, const double* a, const double* x, const
 }
 
 
-sg_status trie_d10n11_b_c384(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
-  sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 384, 1, 9, 9>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 384, 1, 10, 10>(L, a, x, p, m, y, s);
-  return st;
-}
-
-sg_status trie_d10n11_b_c192(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
-  sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 192, 2, 9, 9>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 192, 2, 10, 10>(L, a, x, p, m, y, s);
-  return st;
-}
-
 }  // namespace sg

@@ -11,9 +11,4 @@ sg_status trie_d20n6(const Layout& L, const double* a, const double* x, const ui
   return st;
 }
 
-// without the level-0 suffix products (S0 off; SG_TRIE_VAR=Z, for comparison)
-sg_status trie_d20n6_nos0(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
-  return trie::launch_range<double, 20, 6, 128, 3, 0, 5>(L, a, x, p, m, y, s);
-}
-
 }  // namespace sg

@@ -1,0 +1,36 @@
+// eval_exp.cu -- EXPERIMENT variants of the evaluation kernel, compiled only into libsg_exp.so
+// (build.py --exp; never into the product libsg.so).  Selected at run time by SG_EXP_VAR; used by
+// scripts/gpu_exp.sh to measure what bounds the product kernel.
+#include <stdlib.h>
+#include <string.h>
+
+#include "../eval_trie.cuh"
+
+namespace sg {
+
+// GO: gather-only (all hat values 1; same addresses, loads and Horner adds), cfg3 shape
+template <int MINB>
+static sg_status d10_go(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
+                        cudaStream_t s) {
+  sg_status st = SG_OK;
+#define SG_R(J0, J1) \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB, J0, J1, 0, false, 3, false, 0, 4, 0, false, false, true>(L, a, x, p, m, y, s);
+  SG_R(0, 6) SG_R(7, 7) SG_R(8, 8) SG_R(9, 9) SG_R(10, 10)
+#undef SG_R
+  return st;
+}
+
+// returns true if an experiment variant handled the call
+bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
+                  sg_dtype dt, cudaStream_t s, sg_status* st) {
+  const char* v = getenv("SG_EXP_VAR");
+  if (!v || dt != SG_F64 || L.d != 10 || L.n != 11) return false;
+  const double* a = (const double*)alpha;
+  const double* xx = (const double*)x;
+  double* yy = (double*)y;
+  if (!strcmp(v, "GO3")) { *st = d10_go<3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "GO4")) { *st = d10_go<4>(L, a, xx, perm, m, yy, s); return true; }
+  return false;
+}
+
+}  // namespace sg

@@ -154,7 +154,7 @@ __global__ void __launch_bounds__(kThreads) k_hier_family2(int n, const uint32_t
   (void)E;
 }
 
-sg_status hier_table(sg_grid_s* g, HierTab* tab, cudaStream_t s) {
+sg_status hier_table(const sg_grid_s* g, HierTab* tab) {
   const Layout& L = g->L;
   const int d = L.d, n = L.n;
   tab->F = (d == 1) ? 1 : L.C(d - 1, n - 2);
@@ -162,20 +162,41 @@ sg_status hier_table(sg_grid_s* g, HierTab* tab, cudaStream_t s) {
   uint64_t nb = 0;
   for (int sp = 0; sp <= n - 2; ++sp) nb += (d == 1 ? (sp == 0 ? 1 : 0) : L.C(d - 2, sp)) * (uint64_t)(n - sp);
   tab->nbase = nb;
-  if (!g->d_hier_tab) {
-    const size_t bytes = (size_t)d * (tab->F * 2 * sizeof(uint32_t) + nb * sizeof(uint64_t));
-    cudaError_t e = cudaMalloc(&g->d_hier_tab, bytes);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(hierarchization tables)");
-    uint64_t* b = (uint64_t*)g->d_hier_tab;
-    uint32_t* in = (uint32_t*)(b + (size_t)d * nb);
-    for (int t = 0; t < d; ++t) {
-      const unsigned blocks = (unsigned)((tab->F + kThreads - 1) / kThreads);
-      k_hier_table<<<blocks, kThreads, 0, s>>>(g->d_L, t, tab->F, in + (size_t)t * tab->F * 2, b + (size_t)t * nb);
-      sg_status st = launched("k_hier_table");
-      if (st != SG_OK) return st;
+  void* tabs = g->d_hier_tab.load(std::memory_order_acquire);
+  if (!tabs) {
+    std::lock_guard<std::mutex> lk(g->hier_mu);
+    tabs = g->d_hier_tab.load(std::memory_order_acquire);
+    if (!tabs) {
+      // built on a private stream and synchronised before publishing: a later
+      // call on any other stream must never see half-written tables
+      const size_t bytes = (size_t)d * (tab->F * 2 * sizeof(uint32_t) + nb * sizeof(uint64_t));
+      cudaStream_t bs;
+      cudaError_t e = cudaStreamCreateWithFlags(&bs, cudaStreamNonBlocking);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate(hierarchization tables)");
+      e = cudaMalloc(&tabs, bytes);
+      if (e != cudaSuccess) {
+        cudaStreamDestroy(bs);
+        return cuda_fail(e, "cudaMalloc(hierarchization tables)");
+      }
+      uint64_t* b = (uint64_t*)tabs;
+      uint32_t* in = (uint32_t*)(b + (size_t)d * nb);
+      sg_status st = SG_OK;
+      for (int t = 0; t < d && st == SG_OK; ++t) {
+        const unsigned blocks = (unsigned)((tab->F + kThreads - 1) / kThreads);
+        k_hier_table<<<blocks, kThreads, 0, bs>>>(g->d_L, t, tab->F, in + (size_t)t * tab->F * 2, b + (size_t)t * nb);
+        st = launched("k_hier_table");
+      }
+      e = cudaStreamSynchronize(bs);
+      cudaStreamDestroy(bs);
+      if (st == SG_OK && e != cudaSuccess) st = cuda_fail(e, "cudaStreamSynchronize(hierarchization tables)");
+      if (st != SG_OK) {
+        cudaFree(tabs);
+        return st;
+      }
+      g->d_hier_tab.store(tabs, std::memory_order_release);
     }
   }
-  tab->base = (uint64_t*)g->d_hier_tab;
+  tab->base = (uint64_t*)tabs;
   tab->info = (uint32_t*)(tab->base + (size_t)d * nb);
   return SG_OK;
 }
@@ -229,11 +250,11 @@ sg_status hierarchize_t(const sg_grid_s* g, T* v, cudaStream_t s) {
   const size_t static_smem = sizeof(Layout) + sizeof(FamilyInfo) + 64;
   if (fam_bytes + static_smem <= (size_t)max_smem) {
     HierTab tab;
-    sg_status st = hier_table(const_cast<sg_grid_s*>(g), &tab, s);
+    sg_status st = hier_table(g, &tab);
     if (st != SG_OK) return st;
-    cudaError_t e = cudaFuncSetAttribute(k_hier_family2<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)fam_bytes);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_hier_family2)");
+    static std::atomic<uint64_t> attr_done{0};
+    st = set_smem_attr(k_hier_family2<T>, attr_done, fam_bytes, -1, "cudaFuncSetAttribute(k_hier_family2)");
+    if (st != SG_OK) return st;
     if (tab.F > 0x7fffffffull) return SG_ERR_OVERFLOW;
     for (int t = 0; t < d; ++t) {
       k_hier_family2<T><<<(unsigned)tab.F, kThreads, fam_bytes, s>>>(n, tab.info + (size_t)t * tab.F * 2,

@@ -10,8 +10,6 @@
 // (key, query index) pairs on the caller's stream.
 #include <cub/device/device_radix_sort.cuh>
 
-#include <stdlib.h>
-
 #include "common.cuh"
 
 namespace sg {
@@ -84,7 +82,7 @@ size_t sfc_workspace_bytes(uint64_t m) {
 }
 
 sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dtype dt, void* ws, size_t ws_bytes,
-                           const uint32_t** perm_out, cudaStream_t s) {
+                           uint32_t* perm_dst, const uint32_t** perm_out, cudaStream_t s) {
   if (m > 0x7fffffffull) {
     set_error("sg_evaluate: m = %llu exceeds 2^31-1 queries per call", (unsigned long long)m);
     return SG_ERR_ARG;
@@ -105,14 +103,12 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
   size_t temp = cub_temp_bytes(m);
   const int d = g->L.d, bits = morton_bits(d);
   // lag cap 1: measured best at cfg3 (d = 10, m = 10^7: 7.01-7.05e6 evals/s vs 6.92e6 at caps 2-6 and
-  // 6.94e6 at 0, profiles/r01_v5_variants.txt); SG_MORTON_LAGCAP overrides it (experiment switch)
-  static const char* capenv = getenv("SG_MORTON_LAGCAP");
-  const int cap = capenv ? atoi(capenv) : (bits / 2 < 1 ? bits / 2 : 1);
+  // 6.94e6 at 0, profiles/r01_v5_variants.txt)
+  const int cap = bits / 2 < 1 ? bits / 2 : 1;
   // lag(t) = min(cap, t - start) for t > start; start = d / 2 + 1: measured best at cfg3 (d = 10: dimensions
   // 7-9 one plane late, 7.08e6 evals/s vs 6.88 / 6.97 / 6.99-7.01 / 7.01e6 at start 3 / 4 / 5 / 7,
-  // profiles/r01_v5_variants.txt); SG_MORTON_LAGSTART overrides it (experiment switch)
-  static const char* startenv = getenv("SG_MORTON_LAGSTART");
-  const int start = d < 4 ? d : (startenv ? atoi(startenv) : d / 2 + 1);
+  // profiles/r01_v5_variants.txt)
+  const int start = d < 4 ? d : d / 2 + 1;
   uint64_t blocks = (m + kThreads - 1) / kThreads;
   if (blocks > (uint64_t)kNumSMs * 32) blocks = (uint64_t)kNumSMs * 32;
   if (dt == SG_F64)
@@ -121,9 +117,12 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
     k_morton<float><<<(unsigned)blocks, kThreads, 0, s>>>((const float*)x, m, d, bits, cap, start, k0, v0);
   sg_status st = launched("k_morton");
   if (st != SG_OK) return st;
-  cudaError_t e = cub::DeviceRadixSort::SortPairs(p, temp, k0, k1, v0, v1, (int)m, 0, d * bits, s);
+  // the sort is deterministic (stable LSD radix sort of (key, index) pairs): every rank that orders the same
+  // batch gets the same permutation (ranks agree on one global order without communicating)
+  uint32_t* vout = perm_dst ? perm_dst : v1;
+  cudaError_t e = cub::DeviceRadixSort::SortPairs(p, temp, k0, k1, v0, vout, (int)m, 0, d * bits, s);
   if (e != cudaSuccess) return cuda_fail(e, "cub::DeviceRadixSort::SortPairs");
-  *perm_out = v1;
+  if (perm_out) *perm_out = vout;
   return SG_OK;
 }
 

@@ -42,11 +42,33 @@ ProfScope::ProfScope(int kind_, cudaStream_t s_) : s(s_), kind(kind_) {
   cudaEventRecord(a, s);
 }
 
+// fold finished event pairs into the totals (caller holds g_prof_mu)
+static cudaError_t prof_fold(size_t keep) {
+  cudaError_t st = cudaSuccess;
+  const size_t n = g_prof_pending.size() > keep ? g_prof_pending.size() - keep : 0;
+  for (size_t k = 0; k < n; ++k) {
+    ProfRec& r = g_prof_pending[k];
+    cudaError_t e = cudaEventSynchronize(r.b);
+    float ms = 0.f;
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, r.a, r.b);
+    if (e != cudaSuccess) st = e;
+    g_prof_ms[r.kind] += ms;
+    g_prof_n[r.kind] += 1;
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
+  g_prof_pending.erase(g_prof_pending.begin(), g_prof_pending.begin() + n);
+  return st;
+}
+
 ProfScope::~ProfScope() {
   if (!a) return;
   cudaEventRecord(b, s);
   std::lock_guard<std::mutex> lk(g_prof_mu);
   g_prof_pending.push_back({a, b, kind});
+  // bounded: beyond kProfMax outstanding pairs the oldest half is resolved (profiling mode only)
+  constexpr size_t kProfMax = 4096;
+  if (g_prof_pending.size() > kProfMax) prof_fold(kProfMax / 2);
 }
 
 sg_status cuda_fail(cudaError_t e, const char* what) {
@@ -176,7 +198,7 @@ sg_status sg_destroy(sg_grid g) {
     DeviceGuard guard(g->device);
     cudaDeviceSynchronize();
     cudaFree(g->d_L);
-    if (g->d_hier_tab) cudaFree(g->d_hier_tab);
+    if (void* t = g->d_hier_tab.load()) cudaFree(t);
   }
   delete g;
   return SG_OK;
@@ -292,11 +314,67 @@ sg_status sg_evaluate(sg_grid g, const void* d_alpha, const void* d_x, uint64_t 
       d_workspace = own_ws;
       ws_bytes = need;
     }
-    st = launch_sfc_order(g, d_x, m, dt, d_workspace, ws_bytes, &perm, s);
+    st = launch_sfc_order(g, d_x, m, dt, d_workspace, ws_bytes, nullptr, &perm, s);
   }
   if (st == SG_OK) st = launch_evaluate(g, d_alpha, d_x, perm, m, d_y, dt, flags, s);
   if (own_ws) cudaFreeAsync(own_ws, s);
   return st;
+}
+
+sg_status sg_sfc_order(sg_grid g, const void* d_x, uint64_t m, sg_dtype dt, uint32_t* d_perm, void* d_workspace,
+                       size_t ws_bytes, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (m == 0) return SG_OK;
+  if (!d_x || !d_perm) {
+    set_error("sg_sfc_order: NULL buffer");
+    return SG_ERR_ARG;
+  }
+  if (m > 0x7fffffffull) {
+    set_error("sg_sfc_order: at most 2^31-1 queries per call (got %llu)", (unsigned long long)m);
+    return SG_ERR_ARG;
+  }
+  DeviceGuard guard(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  void* own_ws = nullptr;
+  if (!d_workspace) {
+    ws_bytes = sfc_workspace_bytes(m);
+    cudaError_t e = cudaMallocAsync(&own_ws, ws_bytes, s);
+    if (e != cudaSuccess) return cuda_fail(e, "sg_sfc_order: cudaMallocAsync(workspace)");
+    d_workspace = own_ws;
+  }
+  sg_status st = launch_sfc_order(g, d_x, m, dt, d_workspace, ws_bytes, d_perm, nullptr, s);
+  if (own_ws) cudaFreeAsync(own_ws, s);
+  return st;
+}
+
+sg_status sg_evaluate_ordered(sg_grid g, const void* d_alpha, const void* d_x, uint64_t m, const uint32_t* d_perm,
+                              uint64_t first, uint64_t count, void* d_y, sg_dtype dt, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (first > m || count > m - first) {
+    set_error("sg_evaluate_ordered: range [%llu, +%llu) exceeds m=%llu", (unsigned long long)first,
+              (unsigned long long)count, (unsigned long long)m);
+    return SG_ERR_RANGE;
+  }
+  if (count == 0) return SG_OK;
+  if (!d_alpha || !d_x || !d_y) {
+    set_error("sg_evaluate_ordered: NULL buffer");
+    return SG_ERR_ARG;
+  }
+  if (m > 0x7fffffffull) {
+    set_error("sg_evaluate_ordered: at most 2^31-1 queries per batch (got %llu)", (unsigned long long)m);
+    return SG_ERR_ARG;
+  }
+  DeviceGuard guard(g->device);
+  const size_t es = dtype_size(dt);
+  if (d_perm)  // positions first..first+count-1 of the order; x and y indexed by the query's input position
+    return launch_evaluate(g, d_alpha, d_x, d_perm + first, count, d_y, dt, SG_EVAL_PRESORTED, (cudaStream_t)stream);
+  // no order: the batch is taken as presorted, rows first..first+count-1
+  return launch_evaluate(g, d_alpha, (const char*)d_x + first * (size_t)g->L.d * es, nullptr, count,
+                         (char*)d_y + first * es, dt, SG_EVAL_PRESORTED, (cudaStream_t)stream);
 }
 
 sg_status sg_evaluate_host(sg_grid g, const void* d_alpha, const void* h_x, uint64_t m, void* h_y, sg_dtype dt,
@@ -342,18 +420,8 @@ sg_status sg_profile_enable(int on) {
 sg_status sg_profile_read(double* eval_ms, uint64_t* eval_launches, double* hier_ms, uint64_t* hier_launches,
                           int reset) {
   std::lock_guard<std::mutex> lk(g_prof_mu);
-  sg_status st = SG_OK;
-  for (auto& r : g_prof_pending) {
-    cudaError_t e = cudaEventSynchronize(r.b);
-    float ms = 0.f;
-    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, r.a, r.b);
-    if (e != cudaSuccess) st = cuda_fail(e, "sg_profile_read");
-    g_prof_ms[r.kind] += ms;
-    g_prof_n[r.kind] += 1;
-    cudaEventDestroy(r.a);
-    cudaEventDestroy(r.b);
-  }
-  g_prof_pending.clear();
+  const cudaError_t e = prof_fold(0);
+  const sg_status st = e == cudaSuccess ? SG_OK : cuda_fail(e, "sg_profile_read");
   if (eval_ms) *eval_ms = g_prof_ms[kProfEval];
   if (eval_launches) *eval_launches = g_prof_n[kProfEval];
   if (hier_ms) *hier_ms = g_prof_ms[kProfHier];

@@ -65,7 +65,8 @@ class Grid:
 
     # ---- compression (a7)
     def hierarchize_(self, values: torch.Tensor) -> torch.Tensor:
-        assert values.numel() == self.num_points
+        if values.numel() != self.num_points:
+            raise ValueError(f"values has {values.numel()} entries, the grid {self.num_points} points")
         _sg.sg_hierarchize(self._h, values)
         return values
 
@@ -75,9 +76,26 @@ class Grid:
 
     def evaluate(self, alpha: torch.Tensor, x: torch.Tensor, out: torch.Tensor | None = None,
                  presorted: bool = False, workspace: torch.Tensor | None = None) -> torch.Tensor:
-        assert x.dim() == 2 and x.shape[1] == self.d and x.dtype == alpha.dtype
+        _sg._check_batch(alpha, x, out, self.num_points, self.d)
         y = out if out is not None else torch.empty(x.shape[0], dtype=x.dtype, device=x.device)
         _sg.sg_evaluate(self._h, alpha, x.contiguous(), y, _sg.SG_EVAL_PRESORTED if presorted else 0, workspace)
+        return y
+
+    # ---- the multi-GPU building blocks: one global order, contiguous ranges of it
+    def sfc_order(self, x: torch.Tensor, workspace: torch.Tensor | None = None) -> torch.Tensor:
+        """Morton order of the batch (int32 permutation on x's device), identical on every rank."""
+        _sg._check_batch(x, x, None, None, self.d)
+        perm = torch.empty(x.shape[0], dtype=torch.int32, device=x.device)
+        _sg.sg_sfc_order(self._h, x.contiguous(), perm, workspace)
+        return perm
+
+    def evaluate_ordered(self, alpha: torch.Tensor, x: torch.Tensor, perm: torch.Tensor | None, first: int,
+                         count: int, out: torch.Tensor | None = None) -> torch.Tensor:
+        """Evaluate positions first..first+count-1 of the order `perm`; out is the whole-batch result vector
+        (input order) of which only those queries' entries are written."""
+        _sg._check_batch(alpha, x, out, self.num_points, self.d)
+        y = out if out is not None else torch.zeros(x.shape[0], dtype=x.dtype, device=x.device)
+        _sg.sg_evaluate_ordered(self._h, alpha, x.contiguous(), perm, first, count, y)
         return y
 
     def evaluate_host(self, alpha: torch.Tensor, x_host, y_host=None, presorted: bool = False):

@@ -1,41 +1,63 @@
-"""Multi-GPU plumbing of the decompression path.
+"""Multi-GPU decompression: one global order, contiguous shards, one broadcast.
 
-Evaluation is embarrassingly parallel over query points: every query costs
-exactly T(d, n) terms, so a static partition balances perfectly -- the
-paper's "static workload distribution".  The only
-exchange is the replication of the surplus array: rank 0 compresses
-(hierarchizes) and ONE broadcast (NCCL over NVLink/NVSwitch on B200; gloo in
-the CPU tests) gives every rank the same 1.02 GB of surpluses.  Outputs stay
-sharded; there is no other collective.
+Evaluation is embarrassingly parallel over query points (Sec. 4.3): every query costs
+exactly T(d, n) terms, so a static partition into equal ranges balances perfectly -- the paper's "static
+workload distribution" (L51).  The path on P ranks:
 
-Weak scaling: rank r owns rows ``[r*m, (r+1)*m)`` of ONE global seeded query
-stream (``sginputs.queries(..., first=r*m)``), so the union over ranks is the
-single-process batch of ``world*m`` queries and results are bitwise
-partition-invariant (each query is evaluated by the same kernel code
-whichever rank owns it; Morton ordering only permutes the work).
+1. rank ``src`` compresses (hierarchizes); ONE broadcast of the surplus array (NCCL over NVLink/NVSwitch
+   on B200, 1.02 GB at cfg3; gloo in the CPU tests) replicates it -- the path's only collective;
+2. every rank orders the WHOLE batch along the Morton curve (``sg_sfc_order``: a deterministic stable
+   radix sort, so all ranks obtain the same permutation without communicating, in ~ms);
+3. rank r evaluates the contiguous range ``partition(m, P, r)`` of that global order
+   (``sg_evaluate_ordered``).  Ranges of one global order keep every rank's warps as compact as on one
+   GPU; per-rank local sorts of index slices would not (6.95 vs 4.86 sectors per gather).
+
+Outputs stay sharded: rank r's result vector holds the values of its range's queries (at their input
+positions).  Every query's value is bitwise the same whichever rank evaluates it (the per-query
+arithmetic order is fixed by the enumeration), so the union over ranks equals one-GPU evaluation.
 """
 from __future__ import annotations
 
 
-def shard_range(m_per_rank: int, rank: int) -> tuple[int, int]:
-    """(first, count) of rank's rows in the global query stream."""
-    if m_per_rank < 0 or rank < 0:
-        raise ValueError("m_per_rank and rank must be >= 0")
-    return rank * m_per_rank, m_per_rank
+def partition(m: int, world: int, rank: int) -> tuple[int, int]:
+    """(first, count) of rank's contiguous range of an m-query order: sizes differ by at most one."""
+    if m < 0 or world < 1 or not 0 <= rank < world:
+        raise ValueError(f"bad partition arguments m={m} world={world} rank={rank}")
+    q, r = divmod(m, world)
+    first = rank * q + min(rank, r)
+    return first, q + (1 if rank < r else 0)
 
 
 def replicate_surpluses(alpha, src: int = 0, group=None):
-    """Broadcast the surplus array from ``src`` to every rank, in place.
-
-    The one collective of the path (north_star: "replicated with one NCCL
-    broadcast").  ``alpha`` is a contiguous tensor on the rank's device (CUDA
-    for NCCL, CPU for gloo)."""
+    """Broadcast the surplus array from ``src`` to every rank, in place (north_star: "replicated with one
+    NCCL broadcast").  ``alpha`` is a contiguous tensor on the rank's device (CUDA for NCCL, CPU or CUDA
+    for gloo)."""
     import torch.distributed as dist
     if not alpha.is_contiguous():
         raise ValueError("alpha must be contiguous")
     if dist.is_initialized() and dist.get_world_size(group) > 1:
         dist.broadcast(alpha, src=src, group=group)
     return alpha
+
+
+def evaluate_distributed(grid, alpha, x, group=None, src: int = 0, out=None, perm=None, broadcast: bool = True):
+    """Evaluate this rank's shard of the batch ``x`` (the WHOLE batch, identical on every rank).
+
+    ``alpha`` is broadcast from ``src`` first (skip with ``broadcast=False`` when it is already
+    replicated); ``perm`` may be passed to reuse an order computed earlier.  Returns
+    ``(y, perm, first, count)``: ``y`` (whole-batch length, input order) holds this rank's values at the
+    positions ``perm[first:first+count]``; other entries are left as they were (zeros if ``out`` is None).
+    """
+    import torch.distributed as dist
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    if broadcast:
+        replicate_surpluses(alpha, src=src, group=group)
+    if perm is None:
+        perm = grid.sfc_order(x)
+    first, count = partition(x.shape[0], world, rank)
+    y = grid.evaluate_ordered(alpha, x, perm, first, count, out=out)
+    return y, perm, first, count
 
 
 def checksum(t) -> int:
