@@ -9,13 +9,16 @@ One step = one pass of the whole hot path over one batch:
       surplus buffer and hierarchizes it (sg_hierarchize);
   e   N > 1: one NCCL broadcast of the 1.02 GB surplus array (the only
       collective of the path);
-  a1-a6 decompression: every rank evaluates its own batch of 10^7 seeded random
-      queries (sg_evaluate: Morton ordering + evaluation kernel + scatter).
-Weak scaling: every rank has its own 10^7-query batch (seed + rank).
-`value` = evaluations of all ranks / max-over-ranks step time.
-`e2e`   = the same step through the host-buffer C-ABI entry (sg_evaluate_host),
-          with the nodal values and queries copied from pinned host memory and
-          the results copied back inside the timed region.
+  a1-a6 decompression: every rank orders the whole 10^7-query batch along one
+      global Morton curve (sg_sfc_order, deterministic) and evaluates the
+      rank's contiguous range of that order (sg_evaluate_ordered).
+Strong scaling (default): ONE batch of 10^7 queries split over
+the ranks; --scaling weak gives every rank its own 10^7-query batch.
+`value` = evaluations of the batch / max-over-ranks step time.
+`e2e`   = the same step through the public API (Grid.hierarchize_ +
+          multi.evaluate_distributed) with the nodal values and queries copied
+          from pinned host memory and the results copied back inside the
+          timed region.
 `roofline` = the evaluation kernel (the dominant one), timed with CUDA events
           on its launching stream inside the library (sg_profile_*).
 `cpu_baseline` = the C oracle (oracle/) on a bounded sample of the same
@@ -57,13 +60,20 @@ def peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
-def workload_config(m_per_gpu, n_gpus):
-    return {"workload": "cfg3: d=10, n=11 sparse grid (127,574,017 fp64 surpluses, function A hierarchized "
-                        "each step), 1e7 uniform random queries per GPU (rows [rank*1e7, (rank+1)*1e7) of the SplitMix64 stream, seed 0x5EED0003), "
-                        "Morton-ordered inside sg_evaluate",
-            "d": CFG["d"], "n": CFG["n"], "num_points": 127574017, "queries_per_gpu": m_per_gpu,
-            "global_batch": m_per_gpu * n_gpus, "parallelism": f"query-partitioned x{n_gpus}, alpha broadcast",
-            "l2": "inputs larger than L2 (1.02 GB surpluses, 0.8 GB queries per GPU); no flush"}
+def workload_config(m_batch, n_gpus, weak=False):
+    split = ("1e7 queries per GPU (rows [rank*1e7, (rank+1)*1e7) of the SplitMix64 stream, seed 0x5EED0003), "
+             "each rank's batch Morton-ordered on its GPU" if weak else
+             "one batch of 1e7 uniform random queries (SplitMix64 stream, seed 0x5EED0003) held by every rank, "
+             "ordered along one global Morton curve (sg_sfc_order, identical on every rank), rank r evaluating "
+             "the r-th contiguous range of that order (sg_evaluate_ordered)")
+    return {"workload": "cfg3: d=10, n=11 sparse grid (127,574,017 fp64 surpluses, function A hierarchized on rank 0 "
+                        "each step and broadcast), " + split,
+            "d": CFG["d"], "n": CFG["n"], "num_points": 127574017,
+            "queries_per_gpu": m_batch if weak else -(-m_batch // n_gpus),
+            "global_batch": m_batch * n_gpus if weak else m_batch,
+            "parallelism": f"query ranges x{n_gpus} of one global order, alpha broadcast" if not weak
+            else f"independent batches x{n_gpus}, alpha broadcast",
+            "l2": "inputs larger than L2 (1.02 GB surpluses, 0.8 GB queries); no flush"}
 
 
 class ClockSampler:
@@ -152,8 +162,8 @@ def run_reference(args, rank, world):
     value = per_step * args.steps / dt
     line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": workload_config(per_step, 1),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": workload_config(CFG["m"], world),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                              "sample": f"{per_step} cfg3 queries per step (of the 1e7-query workload), "
                                        f"random surpluses, oracle/sg_oracle.c or_evaluate"},
@@ -171,7 +181,9 @@ def run_sg(args, rank, world, local_rank):
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     d, n = CFG["d"], CFG["n"]
-    m = args.m or CFG["m"]
+    weak = args.scaling == "weak"
+    m_rank = args.m or CFG["m"]  # weak: queries per rank; strong: the whole batch
+    m_batch = m_rank if weak else (args.m or CFG["m"])
     g = P.Grid(d, n)
     N = g.num_points
 
@@ -182,19 +194,39 @@ def run_sg(args, rank, world, local_rank):
         b = min(N, a + chunk)
         values[a:b] = S.f_A_torch(g.coords(a, b - a, device=dev))
     alpha = torch.empty_like(values)
-    first, _ = multi.shard_range(m, rank)  # rank's rows of the one global query stream
-    x = S.queries_torch(d, m, CFG["seed"], device=dev, first=first)
-    y = torch.empty(m, dtype=torch.float64, device=dev)
-    ws = torch.empty(g.workspace_bytes(m), dtype=torch.uint8, device=dev)
+    # strong: every rank holds the whole seeded batch (rows 0..m-1) and evaluates its range of the one
+    # global Morton order; weak: rank r's own batch is rows [r*m, (r+1)*m) of the stream
+    x = S.queries_torch(d, m_batch, CFG["seed"], device=dev, first=rank * m_batch if weak else 0)
+    y = torch.zeros(m_batch, dtype=torch.float64, device=dev)
+    perm = torch.empty(m_batch, dtype=torch.int32, device=dev)
+    ws = torch.empty(g.workspace_bytes(m_batch), dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
+    ev = {k: (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for k in ("bcast", "order")}
+    acc = {"bcast": 0.0, "order": 0.0}
+    timing = {"on": False}
+
+    def timed(k, fn):
+        if not timing["on"]:
+            return fn()
+        ev[k][0].record(stream)
+        r = fn()
+        ev[k][1].record(stream)
+        ev[k][1].synchronize()
+        acc[k] += ev[k][0].elapsed_time(ev[k][1])
+        return r
 
     def step():
         if rank == 0:
             alpha.copy_(values)
             g.hierarchize_(alpha)
         if world > 1:
-            multi.replicate_surpluses(alpha, src=0)  # the path's one collective
-        g.evaluate(alpha, x, out=y, workspace=ws)
+            timed("bcast", lambda: multi.replicate_surpluses(alpha, src=0))  # the path's one collective
+        timed("order", lambda: P.sg_sfc_order(g.handle, x, perm, ws))
+        if weak:
+            g.evaluate_ordered(alpha, x, perm, 0, m_batch, out=y)
+        else:
+            multi.evaluate_distributed(g, alpha, x, out=y, perm=perm, broadcast=False)
 
     def barrier():
         if world > 1:
@@ -230,22 +262,38 @@ def run_sg(args, rank, world, local_rank):
     P.sg_profile_enable(False)
     clk = clocks.stop() if rank == 0 else None
     ms_per_step = elapsed_ms / args.steps
-    value = m * world / (ms_per_step / 1e3)
+    total_queries = m_batch * world if weak else m_batch
+    value = total_queries / (ms_per_step / 1e3)
+    first, count = (0, m_batch) if weak else multi.partition(m_batch, world, rank)
 
-    # ---- e2e through the host-buffer C ABI
+    # phase breakdown (separate untimed pass with per-phase events; max over ranks)
+    timing["on"] = True
+    step()
+    timing["on"] = False
+    bcast_ms = max_over_ranks(acc["bcast"])
+    order_ms = max_over_ranks(acc["order"])
+    eval_ms_rank = max_over_ranks(prof["eval_ms"] / max(1, args.steps))
+
+    # ---- e2e through the public API: host buffers, copies inside the timed region
     e2e = None
     if not args.no_e2e:
         values_h = values.cpu().pin_memory() if rank == 0 else None
         x_h = x.cpu().pin_memory()
-        y_h = torch.empty(m, dtype=torch.float64, pin_memory=True)
+        y_h = torch.empty(m_batch, dtype=torch.float64, pin_memory=True)
+        x_d = torch.empty_like(x)
+        y_d = torch.zeros_like(y)
 
         def step_e2e():
             if rank == 0:
                 alpha.copy_(values_h, non_blocking=True)
                 g.hierarchize_(alpha)
-            if world > 1:
-                multi.replicate_surpluses(alpha, src=0)
-            g.evaluate_host(alpha, x_h, y_h)  # H2D x, evaluate, D2H y, synchronizes
+            x_d.copy_(x_h, non_blocking=True)
+            if weak:
+                g.evaluate(alpha, x_d, out=y_d, workspace=ws)
+            else:
+                multi.evaluate_distributed(g, alpha, x_d, out=y_d, broadcast=world > 1)
+            y_h.copy_(y_d, non_blocking=True)
+            stream.synchronize()
 
         step_e2e()
         barrier()
@@ -256,10 +304,13 @@ def run_sg(args, rank, world, local_rank):
         ev1.record(stream)
         barrier()
         e2e_ms = max_over_ranks(ev0.elapsed_time(ev1)) / e2e_steps
-        assert torch.equal(y_h, y.cpu()), "e2e results differ from the device path"
-        e2e = {"value": m * world / (e2e_ms / 1e3), "unit": UNIT,
-               "h2d_bytes_per_step": (N * 8 if rank == 0 else 0) + m * d * 8, "d2h_bytes_per_step": m * 8,
-               "ms_per_step": e2e_ms, "steps": e2e_steps}
+        own = perm[first:first + count].long().cpu()
+        assert torch.equal(y_h[own], y.cpu()[own]), "e2e results differ from the device path"
+        e2e = {"value": total_queries / (e2e_ms / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": (N * 8 if rank == 0 else 0) + m_batch * d * 8, "d2h_bytes_per_step": m_batch * 8,
+               "ms_per_step": e2e_ms, "steps": e2e_steps,
+               "path": "Grid.hierarchize_ + multi.evaluate_distributed (sg_sfc_order + sg_evaluate_ordered) "
+                       "between pinned-host copies" if not weak else "Grid.evaluate between pinned-host copies"}
 
     if rank != 0:
         return
@@ -268,19 +319,19 @@ def run_sg(args, rank, world, local_rank):
     pk, pk_src = peaks()
     T = g.num_subspaces
     f_mhz = float(pk.get("sm_max_mhz", 1965.0))
-    eval_ms = prof["eval_ms"] / max(1, prof["eval_launches"])
-    gathered = T * 8 * m  # one fp64 surplus per subspace per query
+    eval_ms = prof["eval_ms"] / max(1, prof["eval_launches"])  # per sg_evaluate_ordered call (rank 0)
+    gathered = T * 8 * count  # one fp64 surplus per subspace per query of this rank's range
     achieved = gathered / (eval_ms / 1e3) / 1e9  # GB/s
     lsu_peak = 148 * 128 * f_mhz * 1e6 / 1e9  # L1/SMEM -> RF, 128 B/clk/SM
     fma = math.comb(n + d, d) - 1
     fp64_peak = 148 * 64 * 2 * f_mhz * 1e6 / 1e12  # TFLOP/s, 64 DFMA/clk/SM
-    fp64_achieved = 2 * fma * m / (eval_ms / 1e3) / 1e12
+    fp64_achieved = 2 * fma * count / (eval_ms / 1e3) / 1e12
     traffic = None
     prof_json = os.path.join(ROOT, "profiles", "eval_kernel_ncu.json")
     if os.path.exists(prof_json):
         with open(prof_json) as f:
             pj = json.load(f)
-        if pj.get("m") == m and pj.get("d") == d and pj.get("n") == n:
+        if pj.get("m") == count and pj.get("d") == d and pj.get("n") == n:
             traffic = pj.get("dram_bytes_per_launch")
     roofline = {"bound": "alu", "pipe": "L1/LSU gather of surpluses (128 B/clk/SM x 148 SMs)",
                 "achieved": achieved, "peak": lsu_peak, "unit": "GB/s", "frac": achieved / lsu_peak,
@@ -304,14 +355,17 @@ def run_sg(args, rank, world, local_rank):
                   "pass": bool(err.max() <= 1e-12)}
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": workload_config(m, world),
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "weak" if weak else "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": workload_config(m_batch, world, weak),
             "clocks": clk, "e2e": e2e, "gpu_launches": int(launches), "roofline": roofline,
             "cpu_baseline": cpu, "parity": parity,
-            "breakdown_ms_per_step": {"evaluate_kernel": eval_ms,
-                                      "hierarchize": prof["hier_ms"] / max(1, args.steps),
+            "breakdown_ms_per_step": {"evaluate_kernel_max_rank": eval_ms_rank,
+                                      "sfc_order_max_rank": order_ms, "broadcast_max_rank": bcast_ms,
+                                      "hierarchize_rank0": prof["hier_ms"] / max(1, args.steps),
                                       "hierarchized_points_per_s": N / (prof["hier_ms"] / max(1, args.steps) / 1e3)
-                                      if prof["hier_ms"] > 0 else None}}
+                                      if prof["hier_ms"] > 0 else None,
+                                      "value_excl_broadcast": total_queries / ((ms_per_step - bcast_ms) / 1e3)}}
     print(json.dumps(line), flush=True)
 
 
@@ -321,7 +375,10 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="sg", choices=["sg", "reference"])
-    ap.add_argument("--m", type=int, default=0, help="queries per GPU (default: cfg3's 1e7)")
+    ap.add_argument("--m", type=int, default=0, help="queries (strong: the whole batch; weak: per GPU); default 1e7")
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="strong (default): one 1e7-query batch split over the GPUs by ranges of its global "
+                         "Morton order; weak: a 1e7-query batch per GPU")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")

@@ -252,8 +252,11 @@ sg_status hierarchize_t(const sg_grid_s* g, T* v, cudaStream_t s) {
     HierTab tab;
     sg_status st = hier_table(g, &tab);
     if (st != SG_OK) return st;
+    // the family size differs per grid: opt in to the device maximum once (a permission only; the
+    // launch's own dynamic size decides occupancy)
     static std::atomic<uint64_t> attr_done{0};
-    st = set_smem_attr(k_hier_family2<T>, attr_done, fam_bytes, -1, "cudaFuncSetAttribute(k_hier_family2)");
+    st = set_smem_attr(k_hier_family2<T>, attr_done, (size_t)max_smem - static_smem, -1,
+                       "cudaFuncSetAttribute(k_hier_family2)");
     if (st != SG_OK) return st;
     if (tab.F > 0x7fffffffull) return SG_ERR_OVERFLOW;
     for (int t = 0; t < d; ++t) {
