@@ -39,7 +39,7 @@ struct Ctx {
   const T* phis;  // shared: [(D-3)][NM][kThreads] hat values of dims >= 3 (this lane's column)
   uint32_t K[D];  // finest cell per dimension
   T ph0[NM], ph1[NM], ph2[NM];
-  T res;
+  double res;  // fp64 also for fp32 storage (long sequential sum over the blocks)
   uint64_t b;  // base offset index3 + index2 of the next subspace (warp-uniform)
   int j;       // current level group
 };
@@ -77,7 +77,7 @@ __device__ __forceinline__ void block(Ctx<T, D, NM>& c, int s3, uint32_t P3, T p
     acc = (D > 2) ? fma(acc1, c.ph2[l2], acc) : acc1;
     asm volatile("" ::: "memory");  // keep at most one row of gathers in flight (register budget)
   }
-  c.res = fma(acc, prod3, c.res);
+  c.res = fma((double)acc, (double)prod3, c.res);
   c.b += (uint64_t)((R + 1) * (R + 2) / 2) << c.j;
 }
 
@@ -156,13 +156,13 @@ __global__ void __launch_bounds__(kThreads, 2)
     for (int l = 0; l < NM; ++l) c.ph2[l] = T(1);
   }
   // (no barrier needed: every lane reads only its own shared-memory column)
-  c.res = T(0);
+  c.res = 0.0;
   c.b = 0;
   for (int j = 0; j < n; ++j) {
     c.j = j;
     Upper<T, D, NM, D - 1>::run(c, j, 0, 0u, T(1));
   }
-  if (active) y[src] = bad ? T(NAN) : c.res;
+  if (active) y[src] = bad ? T(NAN) : (T)c.res;
 }
 
 template <typename T, int D, int NM>

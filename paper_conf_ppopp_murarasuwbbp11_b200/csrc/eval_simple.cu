@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(kThreads) k_eval_simple(const Layout* __restri
       bad |= isnan(xq[t]);
     }
     int32_t l[SG_MAX_D + 1];
-    T res = T(0);
+    double res = 0.0;  // fp64 also for fp32 storage: T sequential terms (reading G13)
     uint64_t base = 0;  // index3 + index2 (Alg. 7 "index2")
     for (int j = 0; j < n; ++j) {
       l[0] = j;  // first(d, j) = (j, 0, ..., 0)   (eq. 3)
@@ -57,7 +57,7 @@ __global__ void __launch_bounds__(kThreads) k_eval_simple(const Layout* __restri
           prod *= hat_cell<T>(xq[t], lt, cell);
           index1 = (index1 << lt) + cell;
         }
-        res += prod * __ldg(alpha + base + index1);
+        res += (double)prod * (double)__ldg(alpha + base + index1);
         base += (uint64_t)1 << j;
         if (k + 1 < cj) {  // Alg. 4 next(l); never applied to last(d, j) (reading G5)
           int t = 0;
@@ -69,7 +69,7 @@ __global__ void __launch_bounds__(kThreads) k_eval_simple(const Layout* __restri
         }
       }
     }
-    if (active) y[src] = bad ? T(NAN) : res;
+    if (active) y[src] = bad ? T(NAN) : (T)res;
   }
 }
 

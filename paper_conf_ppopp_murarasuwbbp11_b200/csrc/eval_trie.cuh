@@ -100,7 +100,8 @@ struct Trie {
     T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
     T xin[2];                 // HREG: x of dimensions 2, 3
     uint32_t K[D];
-    T res;
+    double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
+                 // sequential fp32 accumulation would lose ~sqrt(#blocks) ulps of fp32)
     uint32_t b;  // running subspace base (elements), warp-uniform
   };
 
@@ -263,7 +264,7 @@ struct Trie {
       acc = (NI >= 4) ? fma(acc3, ph3[l3], acc) : acc3;
     }
     }
-    c.res = fma(acc, prod, c.res);
+    c.res = fma((double)acc, (double)prod, c.res);
     c.b += cnt(R, NI) << J;
   }
 
@@ -336,7 +337,7 @@ struct Trie {
       // every level of dimensions t..0 is 0: the single subspace of this
       // sub-trie, cell 0 in each of those dimensions (digits of length 0)
       const T a = ld_surplus<CH>(c.alpha + c.b + P);
-      c.res = fma(a, prod * c.s0[(t - I) * NT], c.res);
+      c.res = fma((double)a, (double)(prod * c.s0[(t - I) * NT]), c.res);
       c.b += 1u << J;
     } else if constexpr (t < I) block<J, B>(c, P, prod);
     else if constexpr (t == I) inner_unrolled<J, B, 0>(c, P, prod, H4 ? c.xs[xrow(I) * NT] : T(0));
@@ -466,7 +467,7 @@ struct Trie {
       const T a = ld_surplus<CH>(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
       acc = fma(a, fabs(r), acc);
     }
-    c.res = fma(acc, prod * c.s0[(t - I) * NT], c.res);
+    c.res = fma((double)acc, (double)(prod * c.s0[(t - I) * NT]), c.res);
     c.b += (uint32_t)(t + 1) << J;
   }
 
@@ -585,13 +586,13 @@ __global__ void __launch_bounds__(NT, MINB)
     }
   }
   // (no barrier: every lane reads only its own shared-memory column)
-  c.res = T(0);
+  c.res = 0.0;
   c.b = b0;
   TR::template groups<J0, J1>(c, n);
   if (active) {
-    T r = c.res;
-    if (accumulate) r += y[src];
-    y[src] = bad ? T(NAN) : r;
+    double r = c.res;
+    if (accumulate) r += (double)y[src];
+    y[src] = bad ? T(NAN) : (T)r;
   }
 }
 
