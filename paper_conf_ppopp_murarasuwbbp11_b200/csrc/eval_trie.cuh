@@ -1,6 +1,6 @@
-// eval_trie.cuh -- the evaluation hot path, v2 (rows a2-a6; Alg. 7).
+// eval_trie.cuh -- the evaluation hot path (rows a2-a6; Alg. 7), specialised on the
+// dimension D, a level bound NM >= n and the level groups of one launch (compile time).
 //
-// Specialised on the dimension D and a level bound NM >= n (compile time).
 // One query per thread; queries Morton-ordered (row a1).  Every lane of a
 // warp runs the SAME enumeration of level vectors in the bijection order
 // (Alg. 3: l_{D-1} slowest, l_1 fastest, l_0 implied by the group),
@@ -23,17 +23,18 @@
 //     computed once per block for s = 0..R (it carries the digits of
 //     dimensions 0 and 1, whose levels are tied through l_0 = R - s), M_row
 //     clears the bits below (l_2 + .. + l_{I-1} + sigma), and X_row holds the
-//     digits of dimensions 2..I-1 and of the outer dimensions (P);
-//   * the address is one IMAD.WIDE (index1 * 8 + block base);
+//     digits of dimensions 2..I-1; the outer dimensions' digits P go into the
+//     block's base pointer;
 //   * the basis product is Horner over the trie (Alg. 7's product of d hat
 //     values): acc_1 += alpha * phi_0(l_0) * phi_1(l_1) per term,
 //     one FMA per row / inner level, one per outer trie node.
 // Cells: k_t(l) = K_t >> (NM-1-l) with K_t = clamp(floor(2^{NM-1} x_t)),
 // exact.  Hat values: 2 min(u, 1-u),
-// u = 2^l x - k_t(l), exact (reading G7).  The hat values of the inner
-// dimensions live in registers, those of dimension I in shared memory
-// ([l][lane], conflict-free); dimensions > I recompute them along their
-// loop (u <- frac(2u), exact for x in [0,1), and still 0 outside).
+// u = 2^l x - k_t(l), exact (reading G7).  The hat values of dimensions 0, 1
+// live in registers, those of dimensions 2, 3 and I in shared memory
+// ([row][lane], conflict-free, read once per block / slab / node);
+// dimensions > I recompute them along their loop (u <- frac(2u), exact for
+// x in [0,1), and still 0 outside).
 #pragma once
 #include "common.cuh"
 #include "eval_common.cuh"
@@ -41,45 +42,37 @@
 namespace sg {
 namespace trie {
 
-// Surplus gather with an L1 cache-eviction hint (CH): 0 = plain ld.global.nc,
-// 1 = L1::no_allocate, 2 = L1::evict_first, 3 = L1::evict_last.
-template <int CH, typename T>
-__device__ __forceinline__ T ld_surplus(const T* p) {
-  if constexpr (CH == 0 || sizeof(T) != 8) {
-    return __ldg(p);
-  } else {
-    double v;
-    if constexpr (CH == 1) asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
-    else if constexpr (CH == 2) asm("ld.global.nc.L1::evict_first.f64 %0, [%1];" : "=d"(v) : "l"(p));
-    else asm("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(p));
-    return (T)v;
-  }
-}
+// Compile-time knobs of an instantiation.  The defaults are the configuration measured best at
+// cfg3 (experiments recorded under profiles/).
+struct Knobs {
+  // level-0 suffix products and budget-1 closed forms for outer sub-tries (pays at high d: cfg5)
+  static constexpr bool S0 = false;
+  // experiment builds only (csrc/exp): gather only -- every hat value 1, no hat table read, the same
+  // surplus gathers, addresses and Horner adds (the memory ceiling of the access stream)
+  static constexpr bool GO = false;
+  // dimension-3 hat value read once per slab (l_3) instead of a per-block register array (fewer
+  // live registers, the same number of shared-memory reads)
+  static constexpr bool LZ3 = false;
+  // dimension I: sub-tries of budget <= FULL emitted straight-line; otherwise a loop whose last
+  // TAIL + 1 (small) blocks are merged into one basic block (more surplus loads in flight)
+  static constexpr int FULL = 4;
+  static constexpr int TAIL = 3;
+};
+struct KnobsS0 : Knobs {
+  static constexpr bool S0 = true;
+};
 
-template <typename T, int D, int NM, int NT, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false, bool GO = false>
+template <typename T, int D, int NM, int NT, class KN>
 struct Trie {
-  // GO (experiment builds only, SG_EXP): "gather only" -- every hat value is 1, no hat tables are read;
-  // the same surplus gathers, addresses and Horner adds, to measure the memory ceiling of the access stream
-  static __device__ __forceinline__ T phs_at(const T* phs, int row) { return GO ? T(1) : phs[row * NT]; }
-  static constexpr int I = D < 4 ? D : 4;  // inner (register) dimensions
+  static constexpr int I = D < 4 ? D : 4;  // inner (block) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
-  // shared memory, [row][lane]: hat values of dimensions 2, 3 (loaded per
-  // block), of dimension I (per outer node), then x of dimensions I+1..D-1
-  // HREG: hat values of dimensions 2, 3 recomputed per block by exact
-  // doubling from x (registers) instead of loaded from shared memory (LDS
-  // use the same L1 data stage as the surplus gathers).  Experiment, off:
-  // ptxas then keeps 4 instead of 13 loads in flight (4.88e6 vs 6.91e6).
-  // CHUNK > 0: two-phase blocks (loads of CHUNK terms, then their Horner
-  // accumulation).  Experiment, off: 15 vs 13 loads in flight at first use
-  // in SASS, but no measurable change (6.87e6 vs 6.91e6 evals/s).
-  static constexpr int SM_IN = HREG ? 0 : 2 * NM;
-  // H4: hat values of dimension I by exact doubling along its loop (like the
-  // dimensions > I) instead of an NM-row shared-memory table; x_I is then row
-  // 0 of the x table (less shared memory, more L1 for the gathers)
-  static constexpr int SM_PH = (O > 0 && !H4) ? NM : 0;
-  static constexpr int SM_X = H4 ? O : (O > 1 ? O - 1 : 0);
-  static constexpr int xrow(int t) { return H4 ? t - I : t - I - 1; }
+  static constexpr bool S0 = KN::S0, GO = KN::GO, LZ3 = KN::LZ3;
+  // shared memory, [row][lane]: hat values of dimensions 2, 3 (read per block / slab), of
+  // dimension I (per dimension-I node), then x of dimensions I+1..D-1
+  static constexpr int SM_IN = 2 * NM;
+  static constexpr int SM_PH = O > 0 ? NM : 0;
+  static constexpr int SM_X = O > 1 ? O - 1 : 0;
+  static constexpr int xrow(int t) { return t - I - 1; }
   // S0: suffix products P0[t] = prod_{u <= t} phi_0(x_u), t = I..D-1, so that a
   // sub-trie whose level budget is exhausted (every level of dimensions t..0
   // is 0: one term, one surplus) costs one gather and one FMA instead of a
@@ -90,6 +83,8 @@ struct Trie {
   // cell k_u(1) in its sign bit; one row per dimension
   static constexpr int SM_RHO = (S0 && O > 0 && NM >= 2) ? D : 0;
   static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X + SM_S0 + SM_RHO) * NT * sizeof(T);
+  static constexpr int kFull = KN::FULL;
+  static constexpr int kTail = KN::TAIL;
 
   struct Ctx {
     const T* __restrict__ alpha;
@@ -98,12 +93,14 @@ struct Trie {
     const T* s0;   // S0: this lane's column of the level-0 suffix products
     const T* rho;  // S0: this lane's column of the signed level-1/level-0 hat ratios
     T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
-    T xin[2];                 // HREG: x of dimensions 2, 3
     uint32_t K[D];
     double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
                  // sequential fp32 accumulation would lose ~sqrt(#blocks) ulps of fp32)
     uint32_t b;  // running subspace base (elements), warp-uniform
   };
+
+  // shared-memory hat value (GO: 1)
+  static __device__ __forceinline__ T phs_at(const T* phs, int row) { return GO ? T(1) : phs[row * NT]; }
 
   static constexpr uint32_t cnt(int R, int NI) {  // subspaces per block = C(R+NI-1, NI-1)
     uint32_t c = 1;
@@ -111,79 +108,11 @@ struct Trie {
     return c;
   }
 
-  // flat term index of a block -> l3 | l2 << 8 | l1 << 16 (subspace order, l3 slowest)
-  static constexpr int dec(int R, int NI, int ci) {
-    int l3 = 0;
-    if (NI >= 4)
-      while (ci >= (int)cnt(R - l3, 3)) { ci -= (int)cnt(R - l3, 3); ++l3; }
-    int l2 = 0;
-    if (NI >= 3)
-      while (ci >= R - l3 - l2 + 1) { ci -= R - l3 - l2 + 1; ++l2; }
-    return l3 | (l2 << 8) | (ci << 16);
-  }
-  template <int J, int R, int NI, int C0, int I>
-  static __device__ __forceinline__ void chunk_load(const T* base, const uint32_t* Cs, uint32_t k2, uint32_t k3,
-                                                    T (&av)[CHUNK > 0 ? CHUNK : 1]) {
-    constexpr int CNT = (int)cnt(R, NI);
-    if constexpr (I < CHUNK && C0 + I < CNT) {
-      constexpr int code = dec(R, NI, C0 + I);
-      constexpr int l3 = code & 255, l2 = (code >> 8) & 255, l1 = code >> 16;
-      constexpr int SG = J - R;
-      constexpr int s = l1 + l2 + l3;
-      const uint32_t X3 = (NI >= 4) ? ((k3 >> (NM - 1 - l3 - SG)) & ~((1u << SG) - 1u)) : 0u;
-      const uint32_t Xr = (NI >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG)) & ~((1u << (l3 + SG)) - 1u)) | X3) : X3;
-      constexpr uint32_t M = 0xffffffffu << (l2 + l3 + SG);
-      uint32_t V;
-      asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
-      const T* p;
-      asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
-      av[I] = __ldg(p + ((uint32_t)(C0 + I) << J));
-      chunk_load<J, R, NI, C0, I + 1>(base, Cs, k2, k3, av);
-    }
-  }
-  static constexpr bool LAZY = false;  // lazy reads of ph2/ph3 measured no better (ptxas in-flight 13.2 vs 15.1)
-  template <int R, int NI, int C0, int I>
-  static __device__ __forceinline__ void chunk_acc(const Ctx& c, const T* ph2, const T* ph3,
-                                                   const T (&av)[CHUNK > 0 ? CHUNK : 1], T& acc, T& acc2, T& acc3) {
-    constexpr int CNT = (int)cnt(R, NI);
-    if constexpr (I < CHUNK && C0 + I < CNT) {
-      constexpr int code = dec(R, NI, C0 + I);
-      constexpr int l3 = code & 255, l2 = (code >> 8) & 255, l1 = code >> 16;
-      constexpr int l0 = R - l1 - l2 - l3;
-      if constexpr (NI >= 2) acc2 = fma(av[I] * c.ph[0][l0], c.ph[NI > 1 ? 1 : 0][l1], acc2);
-      else acc2 = fma(av[I], c.ph[0][l0], acc2);
-      if constexpr (l1 == ((NI >= 2) ? R - l3 - l2 : 0)) {  // end of row (l3, l2)
-        // hat values of dimensions 2, 3 read at the row / slab end (LAZY) or
-        // from the per-block registers
-        const T h2 = (NI >= 3) ? (LAZY ? c.phs[(0 * NM + l2) * NT] : ph2[l2]) : T(1);
-        acc3 = (NI >= 3) ? fma(acc2, h2, acc3) : acc2;
-        acc2 = T(0);
-        if constexpr (l2 == ((NI >= 3) ? R - l3 : 0)) {  // end of slab l3
-          const T h3 = (NI >= 4) ? (LAZY ? c.phs[(1 * NM + l3) * NT] : ph3[l3]) : T(1);
-          acc = (NI >= 4) ? fma(acc3, h3, acc) : acc3;
-          acc3 = T(0);
-        }
-      }
-      chunk_acc<R, NI, C0, I + 1>(c, ph2, ph3, av, acc, acc2, acc3);
-    }
-  }
-  template <int J, int R, int NI, int C0>
-  static __device__ __forceinline__ void chunks(const Ctx& c, const T* base, const uint32_t* Cs, uint32_t k2,
-                                                uint32_t k3, const T* ph2, const T* ph3, T& acc, T& acc2, T& acc3) {
-    if constexpr (R <= J && C0 < (int)cnt(R, NI)) {  // (R > J only in dead instantiations)
-      T av[CHUNK > 0 ? CHUNK : 1];
-      chunk_load<J, R, NI, C0, 0>(base, Cs, k2, k3, av);
-      chunk_acc<R, NI, C0, 0>(c, ph2, ph3, av, acc, acc2, acc3);
-      chunks<J, R, NI, C0 + CHUNK>(c, base, Cs, k2, k3, ph2, ph3, acc, acc2, acc3);
-    }
-  }
-
   // ---------------------------------------------------------------- leaf block
   // Group J, R = J - sigma: every shift below is a compile-time constant.
-  // The block spans the NI innermost dimensions (NI = I, or I - 1 for the
-  // pieces of a split block, whose dimension-(NI) digit is then in P).
-  template <int J, int R, int NI = I>
+  template <int J, int R>
   static __device__ __forceinline__ void block(Ctx& c, uint32_t P, T prod) {
+    constexpr int NI = I;
     constexpr int SG = J - R;  // sigma = sum of the outer levels
     // per-lane block base &alpha[b + P] (P = the outer digits, all below bit SG)
     const T* base = c.alpha + c.b + P;
@@ -203,33 +132,13 @@ struct Trie {
       Cs[s] = hi | lo;
     }
     // hat values of dimensions 2, 3 for levels 0..R, from shared memory
-    T ph2[R + 1], ph3[R + 1];
-    if constexpr (CHUNK > 0 && LAZY) {
-      // read at the row / slab ends (chunk_acc)
-    } else if constexpr (HREG) {
-      T u2 = c.xin[0], u3 = c.xin[1];
+    T ph2[R + 1], ph3[LZ3 ? 1 : R + 1];
 #pragma unroll
-      for (int l = 0; l <= R; ++l) {
-        ph2[l] = (NI >= 3) ? hat_u(u2) : T(1);
-        ph3[l] = (NI >= 4) ? hat_u(u3) : T(1);
-        u2 = dbl_u(u2);
-        u3 = dbl_u(u3);
-      }
-    } else {
-#pragma unroll
-      for (int l = 0; l <= R; ++l) {
-        ph2[l] = (NI >= 3) ? phs_at(c.phs, 0 * NM + l) : T(1);
-        ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
-      }
+    for (int l = 0; l <= R; ++l) {
+      ph2[l] = (NI >= 3) ? phs_at(c.phs, 0 * NM + l) : T(1);
+      if constexpr (!LZ3) ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
     }
     T acc = T(0);
-    if constexpr (CHUNK > 0) {
-      // two phases per chunk of CHUNK terms (flat term index in subspace
-      // order): all loads of the chunk first, then the Horner accumulation,
-      // so that the scheduler keeps the whole chunk of loads in flight
-      T acc2 = T(0), acc3 = T(0);
-      chunks<J, R, NI, 0>(c, base, Cs, k2, k3, ph2, ph3, acc, acc2, acc3);
-    } else {
     constexpr int R3 = (NI >= 4) ? R : 0;
     int cidx = 0;  // compile-time after unrolling: rank of the term inside the block
 #pragma unroll
@@ -254,45 +163,36 @@ struct Trie {
           asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
           const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
           asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
-          const T a = ld_surplus<CH>(p + ((uint32_t)cidx << J));
+          const T a = __ldg(p + ((uint32_t)cidx << J));
           if (NI >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[NI > 1 ? 1 : 0][l1], acc2);
           else acc2 = fma(a, c.ph[0][l0], acc2);
           ++cidx;
         }
         acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
       }
-      acc = (NI >= 4) ? fma(acc3, ph3[l3], acc) : acc3;
-    }
+      if constexpr (NI >= 4) {
+        const T h3 = LZ3 ? phs_at(c.phs, 1 * NM + l3) : ph3[LZ3 ? 0 : l3];
+        acc = fma(acc3, h3, acc);
+      } else {
+        acc = acc3;
+      }
     }
     c.res = fma((double)acc, (double)prod, c.res);
     c.b += cnt(R, NI) << J;
   }
 
   // ------------------------------------------------------- outer trie levels
-  // node<J, t, B>: the sub-trie of dimensions t .. 0 whose levels sum to B
+  // node<J, t>: the sub-trie of dimensions t .. 0 whose levels sum to B
   // (l_0 implied), under the outer digits P (dimensions > t, all below bit
-  // J - B) and their hat product `prod`.  B is a compile-time constant at
-  // every node, so every digit shift (J - B for dimension t) is an immediate.
-  // Dimension I (the innermost outer dimension) is emitted as straight-line
-  // code for B <= kFull, and its last kTail + 1 blocks (the small ones, R <=
-  // kTail: 1 + 4 + 10 + 20 terms) are merged into one basic block (kTail = 3
-  // measured 2.8% faster than 2), so that each basic block keeps
-  // more surplus loads in flight (v2 issued one small block at a time and was
-  // latency-bound, profiles/r01_v2_*).  Sub-tries of higher dimensions with at
-  // most FLAT terms can be emitted straight-line too; measured on B200
-  // (profiles/r01_v3_variants.txt) the larger code then thrashes the
-  // instruction cache (23.7% no_instruction stalls at FLAT = 70 vs 14.6% at
-  // FLAT = 0, 6.12e6 vs 6.79e6 evals/s), so FLAT defaults to 0.  SYNC adds a
-  // CTA barrier per dimension-(I+1) node (experiment; slower at 384x1).
-  static constexpr int kFlat = FLAT;  // straight-line sub-trie size (terms)
-  static constexpr int kFull = FULL;  // dimension I: unroll every l_I when B <= kFull
-  static constexpr int kTail = TAIL;  // dimension I: merge the blocks R <= kTail into one basic block
-
-  static constexpr uint32_t binom(int a, int b) {
-    uint32_t c = 1;
-    for (int k = 1; k <= b; ++k) c = c * (uint32_t)(a - b + k) / (uint32_t)k;
-    return c;
-  }
+  // J - B) and their hat product `prod`.  Dimension I (the innermost outer
+  // dimension) is emitted as straight-line code for B <= kFull, and its last
+  // kTail + 1 blocks (the small ones, R <= kTail: 1 + 4 + 10 + 20 terms) are
+  // merged into one basic block (kTail = 3 measured 2.8% faster than 2), so
+  // that each basic block keeps more surplus loads in flight (v2 issued one
+  // small block at a time and was latency-bound, profiles/r01_v2_*).
+  // Straight-line sub-tries of higher dimensions thrash the instruction cache
+  // (23.7% no_instruction stalls at 70 terms, profiles/r01_v3_variants.txt):
+  // only budget-0 sub-tries of dimensions > I are straight-line.
 
   // hat value from u = 2^l x - k(l) (reading G7): max(0, 2 min(u, 1-u))
   static __device__ __forceinline__ T hat_u(T u) {
@@ -308,133 +208,69 @@ struct Trie {
     return u >= T(1) ? u - T(1) : u;
   }
 
-  // dimension I (the innermost outer dimension) at compile-time budget B:
-  // levels l = L .. B unrolled into one basic block
+  // dimension I at compile-time budget B: levels l = L .. B unrolled into one basic block
   template <int J, int B, int L>
-  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod, T u) {
+  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod) {
     if constexpr (L <= B) {
       constexpr int SG = J - B;
-      const T ph = H4 ? hat_u(u) : phs_at(c.phs, SM_IN + L);
+      const T ph = phs_at(c.phs, SM_IN + L);
       const uint32_t kt = c.K[I] >> (NM - 1 - L);
       block<J, B - L>(c, P | (kt << SG), prod * ph);
-      inner_unrolled<J, B, L + 1>(c, P, prod, H4 ? dbl_u(u) : u);
+      inner_unrolled<J, B, L + 1>(c, P, prod);
     }
   }
 
   // sub-trie of dimensions t .. 0 at compile-time budget B, straight-line
-  template <int J, int t, int B, int L>
-  static __device__ __forceinline__ void flat_level(Ctx& c, uint32_t P, T prod, T u) {
-    if constexpr (L <= B) {
-      constexpr int SG = J - B;
-      const uint32_t kt = c.K[t] >> (NM - 1 - L);
-      flat<J, t - 1, B - L>(c, P | (kt << SG), prod * hat_u(u));
-      if constexpr (L < B) flat_level<J, t, B, L + 1>(c, P, prod, dbl_u(u));
-    }
-  }
   template <int J, int t, int B>
   static __device__ __forceinline__ void flat(Ctx& c, uint32_t P, T prod) {
     if constexpr (S0 && B == 0 && t >= I) {
       // every level of dimensions t..0 is 0: the single subspace of this
       // sub-trie, cell 0 in each of those dimensions (digits of length 0)
-      const T a = ld_surplus<CH>(c.alpha + c.b + P);
+      const T a = __ldg(c.alpha + c.b + P);
       c.res = fma((double)a, (double)(prod * c.s0[(t - I) * NT]), c.res);
       c.b += 1u << J;
-    } else if constexpr (t < I) block<J, B>(c, P, prod);
-    else if constexpr (t == I) inner_unrolled<J, B, 0>(c, P, prod, H4 ? c.xs[xrow(I) * NT] : T(0));
-    else flat_level<J, t, B, 0>(c, P, prod, c.xs[xrow(t) * NT]);
-  }
-  template <int t>
-  static constexpr int flat_max() {  // largest budget whose sub-trie at t is straight-line
-    if (t == I) return kFull;
-    int b = 0;
-    while (binom(b + 1 + t, t) <= (uint32_t)kFlat) ++b;
-    return b;
+    } else if constexpr (t < I) {
+      block<J, B>(c, P, prod);
+    } else if constexpr (t == I) {
+      inner_unrolled<J, B, 0>(c, P, prod);
+    } else {
+      static_assert(B == 0, "only budget-0 sub-tries above dimension I are straight-line");
+      // level 0 of dimension t: digit of length 0, hat phi_0(x_t)
+      flat<J, t - 1, 0>(c, P, prod * hat_u(c.xs[xrow(t) * NT]));
+    }
   }
 
-#define SG_TRIE_FLAT(k) \
+#define SG_TRIE_FULL(k) \
   case k:               \
-    if constexpr (k <= FM && k <= J) flat<J, t, (k <= FM && k <= J ? k : 0)>(c, P, prod); \
+    if constexpr (k <= kFull && k <= J) flat<J, I, (k <= kFull && k <= J ? k : 0)>(c, P, prod); \
     break;
-  // dispatch a small run-time budget into the compile-time straight-line sub-tries
-  template <int J, int t>
-  static __device__ __forceinline__ void flat_dispatch(Ctx& c, int B, uint32_t P, T prod) {
-    constexpr int FM = flat_max<t>();
+  // dimension I at a small run-time budget: the compile-time straight-line sub-tries
+  template <int J>
+  static __device__ __forceinline__ void inner_dispatch(Ctx& c, int B, uint32_t P, T prod) {
     switch (B) {
-      SG_TRIE_FLAT(0) SG_TRIE_FLAT(1) SG_TRIE_FLAT(2) SG_TRIE_FLAT(3)
-      SG_TRIE_FLAT(4) SG_TRIE_FLAT(5) SG_TRIE_FLAT(6) SG_TRIE_FLAT(7)
+      SG_TRIE_FULL(0) SG_TRIE_FULL(1) SG_TRIE_FULL(2) SG_TRIE_FULL(3)
+      SG_TRIE_FULL(4) SG_TRIE_FULL(5) SG_TRIE_FULL(6) SG_TRIE_FULL(7)
       default: break;
     }
   }
-#undef SG_TRIE_FLAT
+#undef SG_TRIE_FULL
 
   // tail of dimension I at run-time budget B: the blocks R = RT .. 0
   // (l_I = B - R), merged into one basic block
   template <int J, int RT>
-  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod, T u) {
+  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod) {
     if constexpr (RT >= 0) {
       const int lt = B - RT;
-      const T ph = H4 ? hat_u(u) : phs_at(c.phs, SM_IN + lt);
+      const T ph = phs_at(c.phs, SM_IN + lt);
       const uint32_t kt = c.K[I] >> (NM - 1 - lt);
       block<J, RT>(c, P | (kt << (J - B)), prod * ph);
-      inner_tail<J, RT - 1>(c, B, P, prod, H4 ? dbl_u(u) : u);
+      inner_tail<J, RT - 1>(c, B, P, prod);
     }
-  }
-
-  // Blocks of I = 4 dimensions with R >= kSplit can be split along dimension
-  // 3 into 3-dimensional pieces shared by every R (l_3 at run time, the piece
-  // for budget R - l_3 dispatched by a switch, the last kTail3 + 1 pieces
-  // merged; subspace order kept: l_3 is the slowest of dimensions 0..3, Alg. 3,
-  // P:L373).  This shrinks the code (instruction-cache stalls 4.3% -> 1.6%) but
-  // the smaller basic blocks keep fewer loads in flight: measured at kSplit = 6
-  // 5.99e6 vs 6.70e6 evals/s (profiles/r01_v3_variants.txt), so it is off.
-  static constexpr int kSplit = 16;
-  static constexpr int kTail3 = 2;
-
-#define SG_TRIE_CASE3(r) \
-  case r:                \
-    if constexpr (r <= J) block<J, (r <= J ? r : 0), 3>(c, P, prod); \
-    break;
-  template <int J>
-  static __device__ __forceinline__ void leaf3(Ctx& c, int R, uint32_t P, T prod) {
-    switch (R) {
-      SG_TRIE_CASE3(0) SG_TRIE_CASE3(1) SG_TRIE_CASE3(2) SG_TRIE_CASE3(3)
-      SG_TRIE_CASE3(4) SG_TRIE_CASE3(5) SG_TRIE_CASE3(6) SG_TRIE_CASE3(7)
-      SG_TRIE_CASE3(8) SG_TRIE_CASE3(9) SG_TRIE_CASE3(10) SG_TRIE_CASE3(11)
-      SG_TRIE_CASE3(12) SG_TRIE_CASE3(13) SG_TRIE_CASE3(14) SG_TRIE_CASE3(15)
-      default: break;
-    }
-  }
-#undef SG_TRIE_CASE3
-
-  // pieces l_3 = R - RT .. R of a split block (compile-time), one basic block
-  template <int J, int R, int RT>
-  static __device__ __forceinline__ void tail3(Ctx& c, uint32_t P, T prod) {
-    if constexpr (RT >= 0) {
-      constexpr int l3 = R - RT;
-      const T ph = phs_at(c.phs, 1 * NM + l3);
-      const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
-      block<J, RT, 3>(c, P | (k3 << (J - R)), prod * ph);
-      tail3<J, R, RT - 1>(c, P, prod);
-    }
-  }
-
-  template <int J, int R>
-  static __device__ __forceinline__ void split4(Ctx& c, uint32_t P, T prod) {
-    static_assert(!HREG, "split blocks read the dimension-3 hat table");
-    for (int l3 = 0; l3 < R - kTail3; ++l3) {
-      const T ph = phs_at(c.phs, 1 * NM + l3);
-      const uint32_t k3 = c.K[3] >> (NM - 1 - l3);
-      leaf3<J>(c, R - l3, P | (k3 << (J - R)), prod * ph);
-    }
-    tail3<J, R, kTail3>(c, P, prod);
   }
 
 #define SG_TRIE_CASE(r) \
   case r:               \
-    if constexpr (r <= J) {                                        \
-      if constexpr (I == 4 && r >= kSplit) split4<J, (r <= J ? r : 0)>(c, P, prod); \
-      else block<J, (r <= J ? r : 0)>(c, P, prod);                 \
-    }                                                              \
+    if constexpr (r <= J) block<J, (r <= J ? r : 0)>(c, P, prod); \
     break;
   template <int J>
   static __device__ __forceinline__ void leaf(Ctx& c, int R, uint32_t P, T prod) {
@@ -452,19 +288,17 @@ struct Trie {
   // dimension u (u = 0..t, in the bijection order, Alg. 3: u = 0 first) and
   // every other level of dimensions t..0 zero are consecutive; dimension u's
   // one-bit digit k_u(1) sits just above the outer digits P (bit J - 1).
-  // Horner over u: acc <- acc * phi_0(x_u) + alpha_u * phi_1(x_u) * prod_{v<u} phi_0(x_v),
-  // so that acc = sum_u alpha_u phi_1(x_u) prod_{v<=t, v!=u} phi_0(x_v)
-  // (Alg. 7's product of hat values).
+  // Their sum sum_u alpha_u phi_1(x_u) prod_{v<=t, v!=u} phi_0(x_v) is
+  // S0[t] * sum_u alpha_u rho_u (Alg. 7's product of hat values).
   template <int J, int t>
   static __device__ __forceinline__ void budget1(Ctx& c, uint32_t P, T prod) {
-    // sum_u alpha_u phi_1(x_u) prod_{v<=t, v!=u} phi_0(x_v) = S0[t] * sum_u alpha_u rho_u
     const T* base = c.alpha + c.b + P;
     T acc = T(0);
 #pragma unroll
     for (int u = 0; u <= t; ++u) {
       const T r = c.rho[u * NT];
       const uint32_t k1 = (uint32_t)__double2hiint((double)r) >> 31;  // k_u(1), the sign bit
-      const T a = ld_surplus<CH>(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
+      const T a = __ldg(base + ((k1 << (J - 1)) + ((uint32_t)u << J)));
       acc = fma(a, fabs(r), acc);
     }
     c.res = fma((double)acc, (double)(prod * c.s0[(t - I) * NT]), c.res);
@@ -475,32 +309,31 @@ struct Trie {
   // t..0 sum to B): a run-time loop over l_t, each child inlined once
   template <int J, int t>
   static __device__ __forceinline__ void node(Ctx& c, int B, uint32_t P, T prod) {
-    if constexpr (S0 && !H4 && I == 4 && t > I && J >= 1 && NM >= 2) {
+    if constexpr (S0 && I == 4 && t > I && J >= 1 && NM >= 2) {
       if (B == 1) {
         budget1<J, t>(c, P, prod);
         return;
       }
     }
-    if (B <= flat_max<t>()) {
-      flat_dispatch<J, t>(c, B, P, prod);
-      return;
-    }
     const int SG = J - B;  // shift of dimension t's digit
     if constexpr (t == I) {
-      T u = H4 ? c.xs[xrow(I) * NT] : T(0);  // u at level lt (H4)
+      if (B <= kFull) {
+        inner_dispatch<J>(c, B, P, prod);
+        return;
+      }
       for (int lt = 0; lt < B - kTail; ++lt) {
-        const T ph = H4 ? hat_u(u) : phs_at(c.phs, SM_IN + lt);
+        const T ph = phs_at(c.phs, SM_IN + lt);
         const uint32_t kt = c.K[I] >> (NM - 1 - lt);
         leaf<J>(c, B - lt, P | (kt << SG), prod * ph);
-        if constexpr (H4) u = dbl_u(u);
       }
-      inner_tail<J, kTail>(c, B, P, prod, u);
+      inner_tail<J, kTail>(c, B, P, prod);
     } else {
+      if (B == 0) {
+        flat<J, t, 0>(c, P, prod);
+        return;
+      }
       T u = c.xs[xrow(t) * NT];
       for (int lt = 0; lt <= B; ++lt) {
-        // SYNC: keep the warps of a CTA on the same sub-trie (shared L1 sectors
-        // and instruction-cache lines); the enumeration is CTA-uniform
-        if constexpr (SYNC && t == I + 1) __syncthreads();
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
         node<J, t - 1>(c, B - lt, P | (kt << SG), prod * hat_u(u));
         u = dbl_u(u);
@@ -524,12 +357,11 @@ struct Trie {
 // One launch evaluates the level groups J0..J1 (compile time) for every
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false, bool GO = false>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, class KN>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
                 int n, uint32_t b0, int accumulate, T* __restrict__ y) {
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0, GO>;
+  using TR = Trie<T, D, NM, NT, KN>;
   constexpr int I = TR::I;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   T* sm = reinterpret_cast<T*>(smem_raw);
@@ -569,16 +401,13 @@ __global__ void __launch_bounds__(NT, MINB)
       const long long bits = __double_as_longlong(r) | ((long long)(c1 & 1u) << 63);
       sm[(TR::SM_IN + TR::SM_PH + TR::SM_X + TR::SM_S0 + t) * NT + tid] = (T)__longlong_as_double(bits);
     }
-    if (t < I || (t == I && !H4)) {
+    if (t <= I) {
 #pragma unroll
       for (int l = 0; l < NM; ++l) {
         uint32_t cell;
-        const T h = GO ? T(1) : hat_cell<T>(xt, l, cell);
+        const T h = KN::GO ? T(1) : hat_cell<T>(xt, l, cell);
         if (t < 2) c.ph[t < 2 ? t : 0][l] = h;
-        else if (t < I) {
-          if constexpr (HREG) c.xin[t - 2 < 2 ? t - 2 : 0] = xt;
-          else sm[((t - 2) * NM + l) * NT + tid] = h;
-        }
+        else if (t < I) sm[((t - 2) * NM + l) * NT + tid] = h;
         else sm[(TR::SM_IN + l) * NT + tid] = h;
       }
     } else {
@@ -596,13 +425,12 @@ __global__ void __launch_bounds__(NT, MINB)
   }
 }
 
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, int FLAT = 0, bool SYNC = false, int TAIL = 3, bool HREG = false,
-          int CHUNK = 0, int FULL = 4, int CH = 0, bool H4 = false, bool S0 = false, bool GO = false>
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, class KN = Knobs>
 sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32_t* perm, uint64_t m, T* y,
                        cudaStream_t s) {
   if (J0 >= L.n) return SG_OK;
-  using TR = Trie<T, D, NM, NT, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0, GO>;
-  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, FLAT, SYNC, TAIL, HREG, CHUNK, FULL, CH, H4, S0, GO>;
+  using TR = Trie<T, D, NM, NT, KN>;
+  auto kern = k_eval_trie<T, D, NM, NT, MINB, J0, J1, KN>;
   const size_t smem = TR::smem_bytes;
   // shared memory only for the per-lane tables: the rest of the 256 KB stays L1
   // for the surplus gathers

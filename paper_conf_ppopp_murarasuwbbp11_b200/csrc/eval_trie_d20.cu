@@ -7,7 +7,7 @@ namespace sg {
 
 sg_status trie_d20n6(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
   sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 20, 6, 128, 3, 0, 5, 0, false, 3, false, 0, 4, 0, false, true>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 20, 6, 128, 3, 0, 5, trie::KnobsS0>(L, a, x, p, m, y, s);
   return st;
 }
 

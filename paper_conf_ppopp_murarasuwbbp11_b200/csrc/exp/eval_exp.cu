@@ -8,25 +8,32 @@
 
 namespace sg {
 
+struct KnobsGO : trie::Knobs {
+  static constexpr bool GO = true;
+};
+struct KnobsLZ3 : trie::Knobs {
+  static constexpr bool LZ3 = true;
+};
+
 // GO: gather-only (all hat values 1; same addresses, loads and Horner adds), cfg3 shape
 template <int MINB>
 static sg_status d10_go(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
                         cudaStream_t s) {
   sg_status st = SG_OK;
 #define SG_R(J0, J1) \
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB, J0, J1, 0, false, 3, false, 0, 4, 0, false, false, true>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB, J0, J1, KnobsGO>(L, a, x, p, m, y, s);
   SG_R(0, 6) SG_R(7, 7) SG_R(8, 8) SG_R(9, 9) SG_R(10, 10)
 #undef SG_R
   return st;
 }
 
 // product kernel at MINB CTAs of NT threads per SM (register cap 65536 / (NT MINB))
-template <int MINB, int NT = 128>
+template <int MINB, int NT = 128, class KN = trie::Knobs>
 static sg_status d10_minb(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
                           cudaStream_t s) {
   sg_status st = SG_OK;
 #define SG_R(J0, J1) \
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, NT, MINB, J0, J1>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, NT, MINB, J0, J1, KN>(L, a, x, p, m, y, s);
   SG_R(0, 6) SG_R(7, 7) SG_R(8, 8) SG_R(9, 9) SG_R(10, 10)
 #undef SG_R
   return st;
@@ -45,10 +52,8 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "GO5")) { *st = d10_go<5>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GO6")) { *st = d10_go<6>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "P4")) { *st = d10_minb<4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "N64M6")) { *st = d10_minb<6, 64>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "N64M7")) { *st = d10_minb<7, 64>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "N32M13")) { *st = d10_minb<13, 32>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "N32M14")) { *st = d10_minb<14, 32>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "LZ3")) { *st = d10_minb<3, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "P4LZ3")) { *st = d10_minb<4, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
 
