@@ -3,7 +3,7 @@
 // bijection order with Alg. 4 next(), identically in every lane
 // (warp-uniform control flow); per term the d hat values and index1 digits
 // are recomputed as in Alg. 7.  This is the correctness baseline and the
-// fallback for shapes the fast kernel (eval_fast.cu) does not cover.
+// fallback for shapes the generic kernel (eval_gen.cuh: d <= 12 or 16, 20; n <= 12) does not cover.
 //
 // Hat value: phi_{l,i}(x) = max(0, 1 - |2^{l+1} x - i|) is computed as
 // 2 * min(u, 1 - u), u = 2^l x - k, k = clamp(floor(2^l x)): the same value

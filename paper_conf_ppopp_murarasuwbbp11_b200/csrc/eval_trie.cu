@@ -1,6 +1,6 @@
 // eval_trie.cu -- dispatch of the v2 evaluation kernel (eval_trie.cuh) by
 // (d, n, dtype); shapes without an instantiation return handled = false and
-// fall through to eval_fast.cu / eval_simple.cu.
+// fall through to eval_gen.cuh (generic run-time-level kernels) / eval_simple.cu.
 #include "common.cuh"
 
 namespace sg {
@@ -37,19 +37,18 @@ sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x,
     const double* a = (const double*)alpha;
     const double* xx = (const double*)x;
     double* yy = (double*)y;
-    if (d == 10 && n == 11) {
+    // each instantiation serves every n up to its level bound (launches of groups >= n are skipped)
+    if (d == 10 && n <= 11) {
       sg_status st = trie_d10n11_a(L, a, xx, perm, m, yy, s);
       if (st != SG_OK) return st;
       return trie_d10n11_b(L, a, xx, perm, m, yy, s);
     }
-    if (d == 2 && n == 3) return trie_d2n3(L, a, xx, perm, m, yy, s);
-    if (d == 5 && n == 8) return trie_d5n8(L, a, xx, perm, m, yy, s);
-    if (d == 5 && n == 10) return trie_d5n10(L, a, xx, perm, m, yy, s);
-    if (d == 20 && n == 6) {
-      return trie_d20n6(L, a, xx, perm, m, yy, s);
-    }
+    if (d == 2 && n <= 3) return trie_d2n3(L, a, xx, perm, m, yy, s);
+    if (d == 5 && n <= 8) return trie_d5n8(L, a, xx, perm, m, yy, s);
+    if (d == 5 && n <= 10) return trie_d5n10(L, a, xx, perm, m, yy, s);
+    if (d == 20 && n <= 6) return trie_d20n6(L, a, xx, perm, m, yy, s);
   } else {
-    if (d == 3 && n == 14) return trie_d3n14f(L, (const float*)alpha, (const float*)x, perm, m, (float*)y, s);
+    if (d == 3 && n <= 14) return trie_d3n14f(L, (const float*)alpha, (const float*)x, perm, m, (float*)y, s);
   }
   *handled = false;
   return SG_OK;

@@ -57,6 +57,12 @@ struct Knobs {
   // TAIL + 1 (small) blocks are merged into one basic block (more surplus loads in flight)
   static constexpr int FULL = 4;
   static constexpr int TAIL = 3;
+  // block budgets R this launch evaluates (the others only advance the running subspace base):
+  // a group can be split into launches by R, so that the launch of the many small blocks needs
+  // the register hat tables of dimensions 0, 1 only up to level RMAX (fewer registers, more warps)
+  // and the launch of the few large ones prunes every sub-trie of budget < RMIN
+  static constexpr int RMIN = 0;
+  static constexpr int RMAX = 64;
 };
 struct KnobsS0 : Knobs {
   static constexpr bool S0 = true;
@@ -85,6 +91,8 @@ struct Trie {
   static constexpr size_t smem_bytes = (size_t)(SM_IN + SM_PH + SM_X + SM_S0 + SM_RHO) * NT * sizeof(T);
   static constexpr int kFull = KN::FULL;
   static constexpr int kTail = KN::TAIL;
+  static constexpr int RMIN = KN::RMIN, RMAX = KN::RMAX;
+  static constexpr int PHN = NM < RMAX + 1 ? NM : RMAX + 1;  // levels of the register hat tables
 
   struct Ctx {
     const T* __restrict__ alpha;
@@ -92,7 +100,7 @@ struct Trie {
     const T* xs;   // this lane's column of the x table of dimensions > I
     const T* s0;   // S0: this lane's column of the level-0 suffix products
     const T* rho;  // S0: this lane's column of the signed level-1/level-0 hat ratios
-    T ph[I < 2 ? I : 2][NM];  // hat values of dimensions 0, 1 (registers)
+    T ph[I < 2 ? I : 2][PHN];  // hat values of dimensions 0, 1 (registers), levels < PHN
     uint32_t K[D];
     double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
                  // sequential fp32 accumulation would lose ~sqrt(#blocks) ulps of fp32)
@@ -112,6 +120,31 @@ struct Trie {
   // Group J, R = J - sigma: every shift below is a compile-time constant.
   template <int J, int R>
   static __device__ __forceinline__ void block(Ctx& c, uint32_t P, T prod) {
+    constexpr int NI = I;
+    if constexpr (R < RMIN || R > RMAX) {  // another launch evaluates this block
+      c.b += cnt(R, NI) << J;
+      return;
+    } else {
+      block_eval<J, R>(c, P, prod);
+    }
+  }
+  // number of subspaces of the sub-trie of dimensions t..0 with level sum B (l_0 implied): C(B+t, t)
+  template <int t>
+  static __device__ __forceinline__ uint32_t nsub(int B) {
+    uint32_t r = 0;
+#pragma unroll
+    for (int b = 0; b < NM; ++b)
+      if (b == B) r = binom_c(b + t, t);
+    return r;
+  }
+  static constexpr uint32_t binom_c(int a, int b) {
+    uint32_t c = 1;
+    for (int k = 1; k <= b; ++k) c = c * (uint32_t)(a - b + k) / (uint32_t)k;
+    return c;
+  }
+
+  template <int J, int R>
+  static __device__ __forceinline__ void block_eval(Ctx& c, uint32_t P, T prod) {
     constexpr int NI = I;
     constexpr int SG = J - R;  // sigma = sum of the outer levels
     // per-lane block base &alpha[b + P] (P = the outer digits, all below bit SG)
@@ -309,6 +342,12 @@ struct Trie {
   // t..0 sum to B): a run-time loop over l_t, each child inlined once
   template <int J, int t>
   static __device__ __forceinline__ void node(Ctx& c, int B, uint32_t P, T prod) {
+    if constexpr (RMIN > 0) {
+      if (B < RMIN) {  // every block of this sub-trie has R <= B < RMIN: another launch's
+        c.b += nsub<t>(B) << J;
+        return;
+      }
+    }
     if constexpr (S0 && I == 4 && t > I && J >= 1 && NM >= 2) {
       if (B == 1) {
         budget1<J, t>(c, P, prod);
@@ -406,7 +445,9 @@ __global__ void __launch_bounds__(NT, MINB)
       for (int l = 0; l < NM; ++l) {
         uint32_t cell;
         const T h = KN::GO ? T(1) : hat_cell<T>(xt, l, cell);
-        if (t < 2) c.ph[t < 2 ? t : 0][l] = h;
+        if (t < 2) {
+          if (l < TR::PHN) c.ph[t < 2 ? t : 0][l < TR::PHN ? l : 0] = h;
+        }
         else if (t < I) sm[((t - 2) * NM + l) * NT + tid] = h;
         else sm[(TR::SM_IN + l) * NT + tid] = h;
       }
@@ -439,7 +480,9 @@ sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32
   const sg_status st = set_smem_attr(kern, attr_done, smem, pct, "cudaFuncSetAttribute(k_eval_trie)");
   if (st != SG_OK) return st;
   const unsigned blocks = (unsigned)((m + NT - 1) / NT);
-  kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, L.n, (uint32_t)L.off[J0], J0 > 0 ? 1 : 0, y);
+  // the first launch of a call (group 0, all budgets) writes y, every later one accumulates
+  const int accumulate = (J0 > 0 || KN::RMIN > 0) ? 1 : 0;
+  kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, L.n, (uint32_t)L.off[J0], accumulate, y);
   return launched("k_eval_trie");
 }
 

@@ -16,12 +16,12 @@ struct KnobsLZ3 : trie::Knobs {
 };
 
 // GO: gather-only (all hat values 1; same addresses, loads and Horner adds), cfg3 shape
-template <int MINB>
+template <int MINB, int NT = 128>
 static sg_status d10_go(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
                         cudaStream_t s) {
   sg_status st = SG_OK;
 #define SG_R(J0, J1) \
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB, J0, J1, KnobsGO>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, NT, MINB, J0, J1, KnobsGO>(L, a, x, p, m, y, s);
   SG_R(0, 6) SG_R(7, 7) SG_R(8, 8) SG_R(9, 9) SG_R(10, 10)
 #undef SG_R
   return st;
@@ -39,6 +39,29 @@ static sg_status d10_minb(const Layout& L, const double* a, const double* x, con
   return st;
 }
 
+// groups split by block budget: the small blocks (R <= RL) at MINB_LO CTAs/SM with register hat
+// tables up to level RL, the large ones (R > RL) at 3 CTAs/SM
+template <int RL>
+struct KLow : trie::Knobs {
+  static constexpr int RMAX = RL;
+};
+template <int RL>
+struct KHigh : trie::Knobs {
+  static constexpr int RMIN = RL + 1;
+};
+template <int RL, int MINB_LO, int MINB_06>
+static sg_status d10_split(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                           double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB_06, 0, 6, KLow<6>>(L, a, x, p, m, y, s);
+#define SG_R(J)                                                                                          \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB_LO, J, J, KLow<RL>>(L, a, x, p, m, y, s); \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, J, J, KHigh<RL>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
+
 // returns true if an experiment variant handled the call
 bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
@@ -52,6 +75,12 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "GO5")) { *st = d10_go<5>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GO6")) { *st = d10_go<6>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "P4")) { *st = d10_minb<4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "GO384")) { *st = d10_go<1, 384>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "P384")) { *st = d10_minb<1, 384>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT5")) { *st = d10_split<5, 4, 3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT5B")) { *st = d10_split<5, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT4")) { *st = d10_split<4, 4, 3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT5L3")) { *st = d10_split<5, 3, 3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LZ3")) { *st = d10_minb<3, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "P4LZ3")) { *st = d10_minb<4, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
   return false;

@@ -10,6 +10,8 @@
 // (key, query index) pairs on the caller's stream.
 #include <cub/device/device_radix_sort.cuh>
 
+#include <stdlib.h>
+
 #include "common.cuh"
 
 namespace sg {
@@ -104,11 +106,17 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
   const int d = g->L.d, bits = morton_bits(d);
   // lag cap 1: measured best at cfg3 (d = 10, m = 10^7: 7.01-7.05e6 evals/s vs 6.92e6 at caps 2-6 and
   // 6.94e6 at 0, profiles/r01_v5_variants.txt)
-  const int cap = bits / 2 < 1 ? bits / 2 : 1;
+  int cap = bits / 2 < 1 ? bits / 2 : 1;
+#ifdef SG_EXP  // experiment builds only (libsg_exp.so): curve shape from the environment
+  if (const char* e = getenv("SG_EXP_LAGCAP")) cap = atoi(e);
+#endif
   // lag(t) = min(cap, t - start) for t > start; start = d / 2 + 1: measured best at cfg3 (d = 10: dimensions
   // 7-9 one plane late, 7.08e6 evals/s vs 6.88 / 6.97 / 6.99-7.01 / 7.01e6 at start 3 / 4 / 5 / 7,
   // profiles/r01_v5_variants.txt)
-  const int start = d < 4 ? d : d / 2 + 1;
+  int start = d < 4 ? d : d / 2 + 1;
+#ifdef SG_EXP
+  if (const char* e = getenv("SG_EXP_LAGSTART")) start = atoi(e);
+#endif
   uint64_t blocks = (m + kThreads - 1) / kThreads;
   if (blocks > (uint64_t)kNumSMs * 32) blocks = (uint64_t)kNumSMs * 32;
   if (dt == SG_F64)

@@ -78,8 +78,24 @@ sg_status cuda_fail(cudaError_t e, const char* what) {
 
 sg_status launch_eval_simple(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                              void* y, sg_dtype dt, cudaStream_t s);
-sg_status launch_eval_fast(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
-                           void* y, sg_dtype dt, cudaStream_t s, bool* handled);
+#define SG_GEN_DECL(part)                                                                                      \
+  bool launch_gen_##part(int d, int n, bool f64, const void* a, const void* x, const uint32_t* p, uint64_t m, \
+                         void* y, cudaStream_t s, sg_status* st);
+SG_GEN_DECL(a) SG_GEN_DECL(b) SG_GEN_DECL(c) SG_GEN_DECL(d)
+#undef SG_GEN_DECL
+
+// the generic run-time-level kernel (eval_gen.cuh): d <= 12, n <= 12; 32-bit offsets
+static sg_status launch_eval_gen(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm,
+                                 uint64_t m, void* y, sg_dtype dt, cudaStream_t s, bool* handled) {
+  *handled = false;
+  const int d = g->L.d, n = g->L.n;
+  if (n > 12 || m > 0xffffffffull || g->L.N >= 0xffffffffull) return SG_OK;
+  sg_status st = SG_OK;
+  const bool f64 = dt == SG_F64;
+  *handled = launch_gen_a(d, n, f64, alpha, x, perm, m, y, s, &st) || launch_gen_b(d, n, f64, alpha, x, perm, m, y, s, &st) ||
+             launch_gen_c(d, n, f64, alpha, x, perm, m, y, s, &st) || launch_gen_d(d, n, f64, alpha, x, perm, m, y, s, &st);
+  return st;
+}
 sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                            void* y, sg_dtype dt, cudaStream_t s, bool* handled);
 
@@ -91,7 +107,7 @@ sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, 
     bool handled = false;
     sg_status st = launch_eval_trie(g, alpha, x, perm, m, y, dt, s, &handled);
     if (handled || st != SG_OK) return st;
-    st = launch_eval_fast(g, alpha, x, perm, m, y, dt, s, &handled);
+    st = launch_eval_gen(g, alpha, x, perm, m, y, dt, s, &handled);
     if (handled || st != SG_OK) return st;
   }
   return launch_eval_simple(g, alpha, x, perm, m, y, dt, s);

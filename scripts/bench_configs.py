@@ -2,6 +2,7 @@
 """Device-timed sg_evaluate / sg_hierarchize throughput for every BASELINE.json config (1 GPU).
 
     python scripts/bench_configs.py [--reps 5] [--only cfg3,cfg5] > profiles/rNN_configs.txt
+    python scripts/bench_configs.py --sweep [--reps 3] > profiles/rNN_sweep.txt
 
 Per config: evaluations/s of sg_evaluate (Morton ordering + evaluation kernels
 + scatter, CUDA events around the call on the current stream, median of
@@ -39,11 +40,39 @@ def timed(fn, reps):
     return statistics.median(a.elapsed_time(b) for a, b in ev)
 
 
+def sweep(reps, f_mhz):
+    """Per-term throughput of sg_evaluate for every d in [1,12], n in [2,12] (random surpluses, source B;
+    10^6 queries, fewer for the largest grids): which kernel serves a shape must not cost more than ~2x
+    of the cfg3 per-term rate."""
+    for d in range(1, 13):
+        for n in range(2, 13):
+            g = P.Grid(d, n)
+            N, T = g.num_points, g.num_subspaces
+            if N >= (1 << 31) or N * 8 > 20e9:
+                g.close()
+                continue
+            m = 1_000_000 if T <= 20_000 else (1 << 18 if T <= 400_000 else 1 << 16)
+            alpha = S.random_surplus_torch(N, seed=7, device="cuda")
+            x = S.queries_torch(d, m, 1234 + d, device="cuda")
+            y = torch.empty(m, dtype=torch.float64, device="cuda")
+            ws = torch.empty(g.workspace_bytes(m), dtype=torch.uint8, device="cuda")
+            ms = timed(lambda: g.evaluate(alpha, x, out=y, workspace=ws), reps)
+            rate = m / (ms / 1e3)
+            print(json.dumps({"d": d, "n": n, "points": N, "terms": T, "queries": m, "evaluate_ms": round(ms, 3),
+                              "evals_per_s": rate, "terms_per_s": rate * T,
+                              "gather_roofline_frac": round(rate * T * 8 / (148 * 128 * f_mhz * 1e6), 4)}), flush=True)
+            g.close()
+            del alpha, x, y, ws
+            torch.cuda.empty_cache()
+
+
 def main():
     reps = int(sys.argv[sys.argv.index("--reps") + 1]) if "--reps" in sys.argv else 5
     pk_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     f_mhz = json.load(open(pk_path)).get("sm_max_mhz", 1965.0) if os.path.exists(pk_path) else 1965.0
     torch.cuda.set_device(0)
+    if "--sweep" in sys.argv:
+        return sweep(reps, f_mhz)
     names = ["cfg1", "cfg2", "cfg2p", "cfg3", "cfg4", "cfg5"]
     if "--only" in sys.argv:
         names = sys.argv[sys.argv.index("--only") + 1].split(",")
