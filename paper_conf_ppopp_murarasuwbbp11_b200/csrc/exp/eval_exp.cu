@@ -80,6 +80,11 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "SPLIT5")) { *st = d10_split<5, 4, 3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT5B")) { *st = d10_split<5, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT4")) { *st = d10_split<4, 4, 3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT4B")) { *st = d10_split<4, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT3")) { *st = d10_split<3, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT2")) { *st = d10_split<2, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT3M5")) { *st = d10_split<3, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SPLIT2M5")) { *st = d10_split<2, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT5L3")) { *st = d10_split<5, 3, 3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LZ3")) { *st = d10_minb<3, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "P4LZ3")) { *st = d10_minb<4, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }

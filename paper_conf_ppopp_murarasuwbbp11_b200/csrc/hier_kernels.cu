@@ -120,38 +120,55 @@ __global__ void __launch_bounds__(kThreads) k_hier_family2(int n, const uint32_t
   if ((int)threadIdx.x < L) base[threadIdx.x] = __ldg(bases + first + threadIdx.x);
   __syncthreads();
   const uint32_t E = ((1u << L) - 1u) << s;  // family size 2^s (2^L - 1)
-  // load block by block: block k holds 2^(s+k) consecutive values (coalesced)
-  for (int k = 0; k < L; ++k) {
-    const uint32_t sz = 1u << (s + k), o = ((1u << k) - 1u) << s;
-    const T* src = v + base[k];
-    for (uint32_t w = threadIdx.x; w < sz; w += blockDim.x) fam[o + w] = src[w];
-  }
-  __syncthreads();
-  const uint32_t lomask = (1u << suf) - 1u;
-  for (int k = 1; k < L; ++k) {  // blocks k >= 1 change; parents live in blocks < k
-    const uint32_t sz = 1u << (s + k), o = ((1u << k) - 1u) << s;
-    T* dst = v + base[k];
-    for (uint32_t w = threadIdx.x; w < sz; w += blockDim.x) {
-      const uint32_t lo = w & lomask;
-      const uint32_t c = (w >> suf) & ((1u << k) - 1u);
-      const uint32_t hi = w >> (suf + k);
-      T vl = T(0), vr = T(0);
-      if (c != 0) {  // left parent at c / 2^k
-        const int b = __ffs(c) - 1;
-        const int kp = k - 1 - b;
-        const uint32_t cp = (c >> b) >> 1;
-        vl = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
+  // Flat index w over the family: block k holds 2^(s+k) consecutive values at w = 2^(s+k) - 2^s
+  // (shared-memory offset = w), i.e. k = floor(log2(w + 2^s)) - s.  v3: every thread first issues
+  // all its loads of the family (independent, one round trip), then stores them to shared memory;
+  // v2 loaded block by block (one round trip per block: latency-bound, long_scoreboard 58%,
+  // profiles/r01_v7_hier_ncu.txt).
+  constexpr int U = 8;
+  const uint32_t two_s = 1u << s;
+  for (uint32_t w0 = 0; w0 < E; w0 += U * blockDim.x) {
+    T val[U];
+#pragma unroll
+    for (int i = 0; i < U; ++i) {
+      const uint32_t w = w0 + i * blockDim.x + threadIdx.x;
+      if (w < E) {
+        const uint32_t p = w + two_s;
+        const int k = 31 - __clz(p) - s;
+        val[i] = v[base[k] + (p - (1u << (s + k)))];
       }
-      if (c + 1 != (1u << k)) {  // right parent at (c+1) / 2^k
-        const int b = __ffs(c + 1) - 1;
-        const int kp = k - 1 - b;
-        const uint32_t cp = ((c + 1) >> b) >> 1;
-        vr = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
-      }
-      dst[w] = fam[o + w] - (vl + vr) / T(2);
+    }
+#pragma unroll
+    for (int i = 0; i < U; ++i) {
+      const uint32_t w = w0 + i * blockDim.x + threadIdx.x;
+      if (w < E) fam[w] = val[i];
     }
   }
-  (void)E;
+  __syncthreads();
+  // every point of blocks k >= 1 from its two 1D parents (blocks < k), written straight to global
+  const uint32_t lomask = (1u << suf) - 1u;
+  for (uint32_t w = two_s + threadIdx.x; w < E; w += blockDim.x) {
+    const uint32_t p = w + two_s;
+    const int k = 31 - __clz(p) - s;
+    const uint32_t wl = p - (1u << (s + k));  // index inside block k
+    const uint32_t lo = wl & lomask;
+    const uint32_t c = (wl >> suf) & ((1u << k) - 1u);
+    const uint32_t hi = wl >> (suf + k);
+    T vl = T(0), vr = T(0);
+    if (c != 0) {  // left parent at c / 2^k
+      const int b = __ffs(c) - 1;
+      const int kp = k - 1 - b;
+      const uint32_t cp = (c >> b) >> 1;
+      vl = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
+    }
+    if (c + 1 != (1u << k)) {  // right parent at (c+1) / 2^k
+      const int b = __ffs(c + 1) - 1;
+      const int kp = k - 1 - b;
+      const uint32_t cp = ((c + 1) >> b) >> 1;
+      vr = fam[(((1u << kp) - 1u) << s) + ((((hi << kp) + cp) << suf) | lo)];
+    }
+    v[base[k] + wl] = fam[w] - (vl + vr) / T(2);
+  }
 }
 
 sg_status hier_table(const sg_grid_s* g, HierTab* tab) {
