@@ -62,6 +62,26 @@ static sg_status d10_split(const Layout& L, const double* a, const double* x, co
   return st;
 }
 
+template <int LO, int HI>
+struct KRange : trie::Knobs {
+  static constexpr int RMIN = LO;
+  static constexpr int RMAX = HI;
+};
+// three launches per group from 7: R <= A at MINB_A, A < R <= B at 4, R > B at 3; groups 0-6 at 4
+template <int A, int B, int MINB_A>
+static sg_status d10_split3(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                            double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLow<6>>(L, a, x, p, m, y, s);
+#define SG_R(J)                                                                                                \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB_A, J, J, KRange<0, A>>(L, a, x, p, m, y, s);     \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, J, J, KRange<A + 1, B>>(L, a, x, p, m, y, s);      \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, J, J, KRange<B + 1, 64>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
+
 // returns true if an experiment variant handled the call
 bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
@@ -85,6 +105,9 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "SPLIT2")) { *st = d10_split<2, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT3M5")) { *st = d10_split<3, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT2M5")) { *st = d10_split<2, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S3W25")) { *st = d10_split3<2, 5, 5>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S3W24")) { *st = d10_split3<2, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S3W14")) { *st = d10_split3<1, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT5L3")) { *st = d10_split<5, 3, 3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LZ3")) { *st = d10_minb<3, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "P4LZ3")) { *st = d10_minb<4, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }

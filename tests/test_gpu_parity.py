@@ -165,6 +165,23 @@ def test_hierarchize_fp32_cfg4_grid(P, torch, oracle):
     np.testing.assert_allclose(got, want, rtol=0, atol=atol)
 
 
+def test_hierarchize_cfg3_bit_exact_vs_oracle(P, torch, oracle):
+    """The full cfg3 compression (127,574,017 points, the bench workload) bit-exact against the oracle's
+    Alg. 1 pole recursion (reading G10: dimensions 0..d-1; x0.5 is exact, so FMA contraction cannot
+    change a bit), on function A plus a non-separable term."""
+    d, n = 10, 11
+    g = P.Grid(d, n)
+    vals = torch.empty(g.num_points, dtype=torch.float64, device="cuda")
+    for a in range(0, g.num_points, 1 << 23):
+        b = min(g.num_points, a + (1 << 23))
+        xc = g.coords(a, b - a)
+        vals[a:b] = S.f_A_torch(xc) + 0.25 * torch.sin(7.0 * xc.sum(1))
+    host = vals.cpu().numpy()
+    got = g.hierarchize_(vals).cpu().numpy()
+    want = oracle.hierarchize(d, n, host)
+    assert np.array_equal(got, want)
+
+
 def test_hierarchize_cfg3_closed_form(P, torch, oracle):
     """Full cfg3 grid (127.6M points) against the closed-form surpluses of the
     cubic function A (pin P5'): every surplus positive, a 10^6 sample exact to
@@ -248,17 +265,19 @@ def separable_dp_torch(torch, d, n, X):
     return poly.sum(1)
 
 
-def closed_form_alpha_A(torch, g, dt):
-    """Exact (closed-form) surpluses of function A for every grid point (P5')."""
+def closed_form_alpha_A(torch, oracle, g, dt):
+    """Exact (closed-form) surpluses of function A for every grid point (P5'), at the (l, i) of every index
+    given by the ORACLE's idx2gp (pinned independently of libsg), computed on the device."""
     d = g.d
     c = (torch.arange(d, dtype=torch.float64, device="cuda") + 1.0) / (2.0 * d + 2.0)
     out = torch.empty(g.num_points, dtype=tdt(torch, dt), device="cuda")
     chunk = 1 << 23
     for a in range(0, g.num_points, chunk):
         b = min(g.num_points, a + chunk)
-        l, i = g.idx2gp(torch.arange(a, b, dtype=torch.int64, device="cuda"))
-        x = i.to(torch.float64) / torch.pow(2.0, l.to(torch.float64) + 1.0)
-        out[a:b] = torch.prod(torch.pow(4.0, -l.to(torch.float64)) * (1.0 - c + 3.0 * c * x), dim=1).to(out.dtype)
+        lo, io = oracle.idx2gp(d, g.n, np.arange(a, b, dtype=np.uint64))
+        l = torch.from_numpy(lo).cuda().to(torch.float64)
+        x = torch.from_numpy(io).cuda().to(torch.float64) / torch.pow(2.0, l + 1.0)
+        out[a:b] = torch.prod(torch.pow(4.0, -l) * (1.0 - c + 3.0 * c * x), dim=1).to(out.dtype)
     return out
 
 
@@ -274,11 +293,11 @@ def test_evaluate_cfg3_full_size(P, torch, oracle):
     y = g.evaluate(alpha, x)
     torch.cuda.synchronize()
     rng = np.random.default_rng(3)
-    samp = np.sort(rng.choice(m, 256, replace=False))
+    samp = np.sort(rng.choice(m, 10_000, replace=False))  # K = 10^4 oracle queries at cfg3
     yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy(), x[torch.from_numpy(samp).cuda()].cpu().numpy())
     check_eval(y.cpu().numpy()[samp], yo, ao, TOL["f64"], "cfg3 oracle sample")
     del alpha
-    exact = closed_form_alpha_A(torch, g, "f64")
+    exact = closed_form_alpha_A(torch, oracle, g, "f64")
     y2 = g.evaluate(exact, x)
     worst = 0.0
     for a in range(0, m, 1 << 21):
@@ -296,7 +315,7 @@ def test_evaluate_cfg3_random_surplus_sample(P, torch, oracle):
     alpha = S.random_surplus_torch(g.num_points, seed=99, device="cuda")
     x = S.queries_torch(d, 20000, 1234, device="cuda")
     y = g.evaluate(alpha, x)
-    samp = np.arange(0, 20000, 157)
+    samp = np.arange(0, 20000, 2)  # 10^4 of the call's queries
     yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy(), x[torch.from_numpy(samp).cuda()].cpu().numpy())
     check_eval(y.cpu().numpy()[samp], yo, ao, TOL["f64"], "cfg3 source B")
 
