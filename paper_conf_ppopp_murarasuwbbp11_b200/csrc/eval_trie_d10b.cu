@@ -1,16 +1,30 @@
-// eval_trie_d10b.cu -- instantiations of the v2 evaluation kernel (eval_trie.cuh) for d = 10, n <= 11 (cfg3), groups 9..10.
-// One launch per level-group range; consecutive launches accumulate into y.
-// Split across files only so that nvcc compiles them in parallel.
+// eval_trie_d10b.cu -- instantiations of the evaluation kernel (eval_trie.cuh) for d = 10, n <= 11 (cfg3),
+// groups 9..10, split by block budget as in eval_trie_d10a.cu.  Split across files only so that nvcc
+// compiles them in parallel.
 #include "eval_trie.cuh"
 
 namespace sg {
 
-sg_status trie_d10n11_b(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y, cudaStream_t s) {
+namespace d10b {
+template <int RL>
+struct KLow : trie::Knobs {
+  static constexpr int RMAX = RL;
+};
+template <int RL>
+struct KHigh : trie::Knobs {
+  static constexpr int RMIN = RL + 1;
+};
+}  // namespace d10b
+
+sg_status trie_d10n11_b(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
+                        cudaStream_t s) {
+  using namespace d10b;
   sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 9, 9>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 10, 10>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 9, 9, KLow<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 9, 9, KHigh<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 10, 10, KLow<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 10, 10, KHigh<4>>(L, a, x, p, m, y, s);
   return st;
 }
-
 
 }  // namespace sg
