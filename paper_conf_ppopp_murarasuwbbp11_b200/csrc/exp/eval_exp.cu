@@ -107,6 +107,8 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "SPLIT2M5")) { *st = d10_split<2, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W25")) { *st = d10_split3<2, 5, 5>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W24")) { *st = d10_split3<2, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S3W46")) { *st = d10_split3<4, 6, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S3W47")) { *st = d10_split3<4, 7, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W14")) { *st = d10_split3<1, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT5L3")) { *st = d10_split<5, 3, 3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LZ3")) { *st = d10_minb<3, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }

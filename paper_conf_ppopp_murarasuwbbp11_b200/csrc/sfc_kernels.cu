@@ -104,9 +104,11 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
   p += align_up(m * 4);
   size_t temp = cub_temp_bytes(m);
   const int d = g->L.d, bits = morton_bits(d);
-  // lag cap 1: measured best at cfg3 (d = 10, m = 10^7: 7.01-7.05e6 evals/s vs 6.92e6 at caps 2-6 and
-  // 6.94e6 at 0, profiles/r01_v5_variants.txt)
-  int cap = bits / 2 < 1 ? bits / 2 : 1;
+  // lag cap 2 (dimensions 7, 8, 9 of 10 one, two, two planes late): measured best at cfg3 once the
+  // evaluation kernel is closer to its memory ceiling (r02: 7.83e6 evals/s at caps 2-4 vs 7.62e6 at cap 1,
+  // profiles/r02_split.txt; the L1 bank-pair model, gives 3.90 vs 4.57 cycles per group-10
+  // gather); r01's cap 1 was best for the latency-bound v7 kernel (profiles/r01_v5_variants.txt)
+  int cap = bits / 2 < 2 ? bits / 2 : 2;
 #ifdef SG_EXP  // experiment builds only (libsg_exp.so): curve shape from the environment
   if (const char* e = getenv("SG_EXP_LAGCAP")) cap = atoi(e);
 #endif
