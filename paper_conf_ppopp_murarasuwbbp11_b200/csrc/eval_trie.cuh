@@ -63,6 +63,9 @@ struct Knobs {
   // and the launch of the few large ones prunes every sub-trie of budget < RMIN
   static constexpr int RMIN = 0;
   static constexpr int RMAX = 64;
+  // hat values of dimensions 2, 3 in registers (levels < PHN) instead of shared-memory rows read per
+  // block: no LDS on the L1 data pipe, more live registers (for launches with a small RMAX)
+  static constexpr bool H23 = false;
 };
 struct KnobsS0 : Knobs {
   static constexpr bool S0 = true;
@@ -72,7 +75,7 @@ template <typename T, int D, int NM, int NT, class KN>
 struct Trie {
   static constexpr int I = D < 4 ? D : 4;  // inner (block) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
-  static constexpr bool S0 = KN::S0, GO = KN::GO, LZ3 = KN::LZ3;
+  static constexpr bool S0 = KN::S0, GO = KN::GO, LZ3 = KN::LZ3, H23 = KN::H23 && D >= 4;
   // shared memory, [row][lane]: hat values of dimensions 2, 3 (read per block / slab), of
   // dimension I (per dimension-I node), then x of dimensions I+1..D-1
   static constexpr int SM_IN = 2 * NM;
@@ -101,6 +104,7 @@ struct Trie {
     const T* s0;   // S0: this lane's column of the level-0 suffix products
     const T* rho;  // S0: this lane's column of the signed level-1/level-0 hat ratios
     T ph[I < 2 ? I : 2][PHN];  // hat values of dimensions 0, 1 (registers), levels < PHN
+    T ph23[H23 ? 2 : 1][H23 ? PHN : 1];  // H23: hat values of dimensions 2, 3 (registers)
     uint32_t K[D];
     double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
                  // sequential fp32 accumulation would lose ~sqrt(#blocks) ulps of fp32)
@@ -168,8 +172,13 @@ struct Trie {
     T ph2[R + 1], ph3[LZ3 ? 1 : R + 1];
 #pragma unroll
     for (int l = 0; l <= R; ++l) {
-      ph2[l] = (NI >= 3) ? phs_at(c.phs, 0 * NM + l) : T(1);
-      if constexpr (!LZ3) ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
+      if constexpr (H23) {
+        ph2[l] = c.ph23[0][H23 ? l : 0];
+        if constexpr (!LZ3) ph3[l] = c.ph23[H23 ? 1 : 0][H23 ? l : 0];
+      } else {
+        ph2[l] = (NI >= 3) ? phs_at(c.phs, 0 * NM + l) : T(1);
+        if constexpr (!LZ3) ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
+      }
     }
     T acc = T(0);
     constexpr int R3 = (NI >= 4) ? R : 0;
@@ -447,6 +456,8 @@ __global__ void __launch_bounds__(NT, MINB)
         const T h = KN::GO ? T(1) : hat_cell<T>(xt, l, cell);
         if (t < 2) {
           if (l < TR::PHN) c.ph[t < 2 ? t : 0][l < TR::PHN ? l : 0] = h;
+        } else if (TR::H23 && t < 4 && l < TR::PHN) {
+          c.ph23[TR::H23 ? t - 2 : 0][TR::H23 && l < TR::PHN ? l : 0] = h;
         }
         else if (t < I) sm[((t - 2) * NM + l) * NT + tid] = h;
         else sm[(TR::SM_IN + l) * NT + tid] = h;

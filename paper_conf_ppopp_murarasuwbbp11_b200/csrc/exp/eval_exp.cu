@@ -82,6 +82,25 @@ static sg_status d10_split3(const Layout& L, const double* a, const double* x, c
   return st;
 }
 
+template <int RL, bool HH, int TL>
+struct KLowX : trie::Knobs {
+  static constexpr int RMAX = RL;
+  static constexpr bool H23 = HH;
+  static constexpr int TAIL = TL;
+};
+template <bool HH, int TL>
+static sg_status d10_splitx(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                            double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLowX<6, HH, 3>>(L, a, x, p, m, y, s);
+#define SG_R(J)                                                                                              \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, J, J, KLowX<4, HH, TL>>(L, a, x, p, m, y, s); \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, J, J, KHigh<4>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
+
 // returns true if an experiment variant handled the call
 bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
@@ -107,6 +126,9 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "SPLIT2M5")) { *st = d10_split<2, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W25")) { *st = d10_split3<2, 5, 5>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W24")) { *st = d10_split3<2, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SXH")) { *st = d10_splitx<true, 3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SXT")) { *st = d10_splitx<false, 4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SXHT")) { *st = d10_splitx<true, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W46")) { *st = d10_split3<4, 6, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W47")) { *st = d10_split3<4, 7, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "S3W14")) { *st = d10_split3<1, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
