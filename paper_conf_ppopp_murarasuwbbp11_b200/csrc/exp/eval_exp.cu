@@ -101,11 +101,38 @@ static sg_status d10_splitx(const Layout& L, const double* a, const double* x, c
   return st;
 }
 
+// cfg5 (d = 20, n = 6, S0 knob): occupancy and block-budget splits
+template <int LO, int HI>
+struct KS0R : trie::KnobsS0 {
+  static constexpr int RMIN = LO;
+  static constexpr int RMAX = HI;
+};
+template <int MINB>
+static sg_status d20_minb(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
+                          cudaStream_t s) {
+  return trie::launch_range<double, 20, 6, 128, MINB, 0, 5, trie::KnobsS0>(L, a, x, p, m, y, s);
+}
+template <int RL, int MINB_LO>
+static sg_status d20_split(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                           double* y, cudaStream_t s) {
+  sg_status st = trie::launch_range<double, 20, 6, 128, MINB_LO, 0, 5, KS0R<0, RL>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 20, 6, 128, 3, 0, 5, KS0R<RL + 1, 64>>(L, a, x, p, m, y, s);
+  return st;
+}
+
 // returns true if an experiment variant handled the call
 bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
   const char* v = getenv("SG_EXP_VAR");
-  if (!v || dt != SG_F64 || L.d != 10 || L.n != 11) return false;
+  if (!v || dt != SG_F64) return false;
+  if (L.d == 20 && L.n == 6) {
+    const double* a = (const double*)alpha;
+    if (!strcmp(v, "D20M4")) { *st = d20_minb<4>(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
+    if (!strcmp(v, "D20S2")) { *st = d20_split<2, 4>(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
+    if (!strcmp(v, "D20S3")) { *st = d20_split<3, 4>(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
+    return false;
+  }
+  if (L.d != 10 || L.n != 11) return false;
   const double* a = (const double*)alpha;
   const double* xx = (const double*)x;
   double* yy = (double*)y;

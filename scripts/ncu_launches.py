@@ -23,9 +23,9 @@ def main(path):
         agg[k][0] += 1
         agg[k][1] += float(r[vi].replace(",", "")) * SCALE.get(r[ui], 1.0)
     tot = sum(a[1] for a in agg.values())
-    print(f"{'kernel':90s} {'launches':>8s} {'total ms':>12s} {'share':>7s}")
+    print(f"{'kernel':120s} {'launches':>8s} {'total ms':>12s} {'share':>7s}")
     for k, (c, t) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
-        print(f"{k[:90]:90s} {c:8d} {t:12.3f} {100 * t / tot:6.2f}%")
+        print(f"{k[:120]:120s} {c:8d} {t:12.3f} {100 * t / tot:6.2f}%")
 
 
 if __name__ == "__main__":
