@@ -169,6 +169,21 @@ sg_status sg_sfc_order(sg_grid g, const void *d_x, uint64_t m, sg_dtype dt, uint
 sg_status sg_evaluate_ordered(sg_grid g, const void *d_alpha, const void *d_x, uint64_t m, const uint32_t *d_perm,
                               uint64_t first, uint64_t count, void *d_y, sg_dtype dt, void *stream);
 
+/* Visualization slice (the paper's motivating application, interactive visualization
+ * of compressed data, Fig. 1; evaluation "at arbitrary locations"): renders
+ * d_image[b * width + a] = f_s(x(a, b)),  x(a, b) = origin + (a + 1/2) du + (b + 1/2) dv,
+ * for pixel columns a < width and rows b < height, each coordinate rounded as
+ * fl(fl(origin_t + (a+1/2) du_t) + (b+1/2) dv_t) in fp64, then converted to dt.  origin, du, dv are HOST
+ * arrays of d doubles (copied at the call).  order 0 visits the pixels in row-major order, order 1 in
+ * 8 x 4 warp tiles along a 2D Morton curve of the tiles (needs width % 8 == 0 and height % 4 == 0, else
+ * row-major).  No query array is needed: the pixel coordinates and the visiting order are generated on the
+ * device into d_workspace (sg_plane_workspace_bytes bytes, or NULL: allocated stream-ordered).  The values
+ * are bitwise those of sg_evaluate at the same points.  Asynchronous. */
+sg_status sg_plane_workspace_bytes(sg_grid g, uint32_t width, uint32_t height, sg_dtype dt, size_t *bytes);
+sg_status sg_evaluate_plane(sg_grid g, const void *d_alpha, const double *origin, const double *du, const double *dv,
+                            uint32_t width, uint32_t height, void *d_image, sg_dtype dt, uint32_t order,
+                            void *d_workspace, size_t ws_bytes, void *stream);
+
 /* End-to-end evaluation from HOST buffers: copies h_x (m x d) to the device,
  * evaluates as sg_evaluate, copies the m results to h_y.  d_alpha is on the
  * device.  Device buffers are allocated stream-ordered.  The three steps run

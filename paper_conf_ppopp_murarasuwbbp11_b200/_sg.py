@@ -55,6 +55,8 @@ _SIGS = {
     "sg_evaluate_host": [_p, _p, _p, _u64, _p, ctypes.c_int, _u32, _p],
     "sg_sfc_order": [_p, _p, _u64, ctypes.c_int, _p, _p, _sz, _p],
     "sg_evaluate_ordered": [_p, _p, _p, _u64, _p, _u64, _u64, _p, ctypes.c_int, _p],
+    "sg_plane_workspace_bytes": [_p, _u32, _u32, ctypes.c_int, ctypes.POINTER(_sz)],
+    "sg_evaluate_plane": [_p, _p, _p, _p, _p, _u32, _u32, _p, ctypes.c_int, _u32, _p, _sz, _p],
 }
 for _name, _args in _SIGS.items():
     _f = getattr(lib, _name)
@@ -222,6 +224,29 @@ def sg_evaluate_ordered(g, alpha: torch.Tensor, x: torch.Tensor, perm: torch.Ten
     pp = _dev(perm, "perm") if perm is not None else None
     _check(lib.sg_evaluate_ordered(g, _dev(alpha, "alpha"), _dev(x, "x"), x.shape[0], pp, first, count, _dev(y, "y"),
                                    _dtype_code(x), _stream(stream)), "sg_evaluate_ordered")
+
+
+def sg_plane_workspace_bytes(g, width: int, height: int, dtype) -> int:
+    b = ctypes.c_size_t()
+    _check(lib.sg_plane_workspace_bytes(g, width, height, _dtype_code(dtype), ctypes.byref(b)),
+           "sg_plane_workspace_bytes")
+    return int(b.value)
+
+
+def sg_evaluate_plane(g, alpha: torch.Tensor, origin, du, dv, image: torch.Tensor, order: int = 1,
+                      workspace: torch.Tensor | None = None, stream=None) -> None:
+    """image (height, width) <- f_s on the plane origin + (a+1/2) du + (b+1/2) dv."""
+    if image.dim() != 2 or image.dtype != alpha.dtype:
+        raise ValueError("image must be a (height, width) tensor of alpha's dtype")
+    h, w = image.shape
+    o = np.ascontiguousarray(origin, dtype=np.float64)
+    u = np.ascontiguousarray(du, dtype=np.float64)
+    v = np.ascontiguousarray(dv, dtype=np.float64)
+    ws = _dev(workspace, "workspace") if workspace is not None else None
+    wsb = workspace.numel() * workspace.element_size() if workspace is not None else 0
+    _check(lib.sg_evaluate_plane(g, _dev(alpha, "alpha"), _np_ptr(o), _np_ptr(u), _np_ptr(v), w, h,
+                                 _dev(image, "image"), _dtype_code(alpha), order, ws, wsb, _stream(stream)),
+           "sg_evaluate_plane")
 
 
 def sg_evaluate_host(g, alpha: torch.Tensor, x_host, y_host, flags: int = 0, stream=None) -> None:

@@ -80,5 +80,9 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
                            uint32_t* perm_dst, const uint32_t** perm_out, cudaStream_t s);
 sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                           void* y, sg_dtype dt, uint32_t flags, cudaStream_t s);
+size_t plane_workspace_bytes(int d, uint64_t m, size_t elem);
+sg_status launch_plane(const sg_grid_s* g, const void* alpha, const double* origin, const double* du, const double* dv,
+                       uint32_t width, uint32_t height, void* img, sg_dtype dt, uint32_t order, void* ws,
+                       cudaStream_t s);
 
 }  // namespace sg

@@ -66,6 +66,12 @@ struct Knobs {
   // hat values of dimensions 2, 3 in registers (levels < PHN) instead of shared-memory rows read per
   // block: no LDS on the L1 data pipe, more live registers (for launches with a small RMAX)
   static constexpr bool H23 = false;
+  // products phi_0(r - l1) phi_1(l1), r <= RMAX, in registers instead of the tables of dimensions 0, 1:
+  // one FMA per term instead of a multiply and an FMA (for launches with a small RMAX)
+  static constexpr bool D01 = false;
+  // inner (block) dimensions: blocks over dimensions 0..INNER-1 (smaller blocks and per-block register
+  // arrays with INNER = 3; dimension 3 then becomes the innermost trie loop)
+  static constexpr int INNER = 4;
 };
 struct KnobsS0 : Knobs {
   static constexpr bool S0 = true;
@@ -73,9 +79,10 @@ struct KnobsS0 : Knobs {
 
 template <typename T, int D, int NM, int NT, class KN>
 struct Trie {
-  static constexpr int I = D < 4 ? D : 4;  // inner (block) dimensions
+  static constexpr int I = D < KN::INNER ? D : KN::INNER;  // inner (block) dimensions
   static constexpr int O = D - I;          // outer (trie) dimensions
   static constexpr bool S0 = KN::S0, GO = KN::GO, LZ3 = KN::LZ3, H23 = KN::H23 && D >= 4;
+  static constexpr bool D01 = KN::D01 && D >= 2;
   // shared memory, [row][lane]: hat values of dimensions 2, 3 (read per block / slab), of
   // dimension I (per dimension-I node), then x of dimensions I+1..D-1
   static constexpr int SM_IN = 2 * NM;
@@ -103,7 +110,8 @@ struct Trie {
     const T* xs;   // this lane's column of the x table of dimensions > I
     const T* s0;   // S0: this lane's column of the level-0 suffix products
     const T* rho;  // S0: this lane's column of the signed level-1/level-0 hat ratios
-    T ph[I < 2 ? I : 2][PHN];  // hat values of dimensions 0, 1 (registers), levels < PHN
+    T ph[I < 2 ? I : 2][D01 ? 1 : PHN];  // hat values of dimensions 0, 1 (registers), levels < PHN
+    T d01[D01 ? PHN * (PHN + 1) / 2 : 1];  // D01: phi_0(r - l1) phi_1(l1) at index r (r + 1) / 2 + l1
     T ph23[H23 ? 2 : 1][H23 ? PHN : 1];  // H23: hat values of dimensions 2, 3 (registers)
     uint32_t K[D];
     double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
@@ -206,8 +214,14 @@ struct Trie {
           const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
           asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
           const T a = __ldg(p + ((uint32_t)cidx << J));
-          if (NI >= 2) acc2 = fma(a * c.ph[0][l0], c.ph[NI > 1 ? 1 : 0][l1], acc2);
-          else acc2 = fma(a, c.ph[0][l0], acc2);
+          if constexpr (D01) {
+            const int r = R - l2 - l3;
+            acc2 = fma(a, c.d01[D01 ? r * (r + 1) / 2 + l1 : 0], acc2);
+          } else if (NI >= 2) {
+            acc2 = fma(a * c.ph[0][D01 ? 0 : l0], c.ph[NI > 1 ? 1 : 0][D01 ? 0 : l1], acc2);
+          } else {
+            acc2 = fma(a, c.ph[0][D01 ? 0 : l0], acc2);
+          }
           ++cidx;
         }
         acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
@@ -429,6 +443,7 @@ __global__ void __launch_bounds__(NT, MINB)
   // dimensions 0..I (registers for 0, 1; shared memory for 2, 3, I)
   bool bad = false;
   const T fine = (T)(1u << (NM - 1));
+  T h01[2][TR::PHN];  // D01: hat values of dimensions 0, 1 before their pairwise products
 #pragma unroll
   for (int t = 0; t < D; ++t) {
     const T xt = active ? x[(size_t)src * D + t] : T(0.5);
@@ -455,7 +470,10 @@ __global__ void __launch_bounds__(NT, MINB)
         uint32_t cell;
         const T h = KN::GO ? T(1) : hat_cell<T>(xt, l, cell);
         if (t < 2) {
-          if (l < TR::PHN) c.ph[t < 2 ? t : 0][l < TR::PHN ? l : 0] = h;
+          if (l < TR::PHN) {
+            if constexpr (TR::D01) h01[t < 2 ? t : 0][l < TR::PHN ? l : 0] = h;
+            else c.ph[t < 2 ? t : 0][l < TR::PHN ? l : 0] = h;
+          }
         } else if (TR::H23 && t < 4 && l < TR::PHN) {
           c.ph23[TR::H23 ? t - 2 : 0][TR::H23 && l < TR::PHN ? l : 0] = h;
         }
@@ -465,6 +483,12 @@ __global__ void __launch_bounds__(NT, MINB)
     } else {
       sm[(TR::SM_IN + TR::SM_PH + TR::xrow(t)) * NT + tid] = xt;
     }
+  }
+  if constexpr (TR::D01) {
+#pragma unroll
+    for (int r = 0; r < TR::PHN; ++r)
+#pragma unroll
+      for (int l1 = 0; l1 <= r; ++l1) c.d01[r * (r + 1) / 2 + l1] = h01[0][r - l1] * h01[1][l1];
   }
   // (no barrier: every lane reads only its own shared-memory column)
   c.res = 0.0;

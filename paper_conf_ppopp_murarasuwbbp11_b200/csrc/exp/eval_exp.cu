@@ -82,12 +82,25 @@ static sg_status d10_split3(const Layout& L, const double* a, const double* x, c
   return st;
 }
 
-template <int RL, bool HH, int TL>
+template <int RL, bool HH, int TL, bool DD = false>
 struct KLowX : trie::Knobs {
   static constexpr int RMAX = RL;
   static constexpr bool H23 = HH;
   static constexpr int TAIL = TL;
+  static constexpr bool D01 = DD;
 };
+template <int RL>
+static sg_status d10_splitd(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                            double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLowX<6, false, 3, false>>(L, a, x, p, m, y, s);
+#define SG_R(J)                                                                                                    \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, J, J, KLowX<RL, false, 3, true>>(L, a, x, p, m, y, s); \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, J, J, KHigh<RL>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
 template <bool HH, int TL>
 static sg_status d10_splitx(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
                             double* y, cudaStream_t s) {
@@ -120,6 +133,25 @@ static sg_status d20_split(const Layout& L, const double* a, const double* x, co
   return st;
 }
 
+template <int RL>
+struct KHigh3 : trie::Knobs {
+  static constexpr int RMIN = RL + 1;
+  static constexpr int INNER = 3;
+};
+// the large-block launch with blocks over dimensions 0..2 (dimension 3 a trie loop), at MINB_HI CTAs/SM
+template <int MINB_HI, bool DD>
+static sg_status d10_splith(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                            double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLowX<6, false, 3, false>>(L, a, x, p, m, y, s);
+#define SG_R(J)                                                                                                    \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, J, J, KLowX<4, false, 3, DD>>(L, a, x, p, m, y, s); \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, MINB_HI, J, J, KHigh3<4>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
+
 // returns true if an experiment variant handled the call
 bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
@@ -138,30 +170,13 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   double* yy = (double*)y;
   if (!strcmp(v, "GO3")) { *st = d10_go<3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GO4")) { *st = d10_go<4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "GO5")) { *st = d10_go<5>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "GO6")) { *st = d10_go<6>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "P4")) { *st = d10_minb<4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "GO384")) { *st = d10_go<1, 384>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "P384")) { *st = d10_minb<1, 384>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT5")) { *st = d10_split<5, 4, 3>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT5B")) { *st = d10_split<5, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT4")) { *st = d10_split<4, 4, 3>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT4B")) { *st = d10_split<4, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT3")) { *st = d10_split<3, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT2")) { *st = d10_split<2, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT3M5")) { *st = d10_split<3, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT2M5")) { *st = d10_split<2, 5, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "S3W25")) { *st = d10_split3<2, 5, 5>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "S3W24")) { *st = d10_split3<2, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SXH")) { *st = d10_splitx<true, 3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SD4")) { *st = d10_splitd<4>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SD3")) { *st = d10_splitd<3>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SH33")) { *st = d10_splith<3, false>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SH34")) { *st = d10_splith<4, false>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SH34D")) { *st = d10_splith<4, true>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SXT")) { *st = d10_splitx<false, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SXHT")) { *st = d10_splitx<true, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "S3W46")) { *st = d10_split3<4, 6, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "S3W47")) { *st = d10_split3<4, 7, 4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "S3W14")) { *st = d10_split3<1, 4, 5>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SPLIT5L3")) { *st = d10_split<5, 3, 3>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "LZ3")) { *st = d10_minb<3, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "P4LZ3")) { *st = d10_minb<4, 128, KnobsLZ3>(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
 

@@ -393,6 +393,47 @@ sg_status sg_evaluate_ordered(sg_grid g, const void* d_alpha, const void* d_x, u
                          (char*)d_y + first * es, dt, SG_EVAL_PRESORTED, (cudaStream_t)stream);
 }
 
+sg_status sg_plane_workspace_bytes(sg_grid g, uint32_t width, uint32_t height, sg_dtype dt, size_t* bytes) {
+  SG_CHECK_GRID(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (!bytes) return SG_ERR_ARG;
+  *bytes = plane_workspace_bytes(g->L.d, (uint64_t)width * height, dtype_size(dt));
+  return SG_OK;
+}
+
+sg_status sg_evaluate_plane(sg_grid g, const void* d_alpha, const double* origin, const double* du, const double* dv,
+                            uint32_t width, uint32_t height, void* d_image, sg_dtype dt, uint32_t order,
+                            void* d_workspace, size_t ws_bytes, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  const uint64_t m = (uint64_t)width * height;
+  if (m == 0) return SG_OK;
+  if (!d_alpha || !origin || !du || !dv || !d_image) {
+    set_error("sg_evaluate_plane: NULL argument");
+    return SG_ERR_ARG;
+  }
+  if (m > 0x7fffffffull || order > 1) {
+    set_error("sg_evaluate_plane: need width*height < 2^31 and order 0 or 1");
+    return SG_ERR_ARG;
+  }
+  DeviceGuard guard(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t need = plane_workspace_bytes(g->L.d, m, dtype_size(dt));
+  void* own = nullptr;
+  if (!d_workspace) {
+    cudaError_t e = cudaMallocAsync(&own, need, s);
+    if (e != cudaSuccess) return cuda_fail(e, "sg_evaluate_plane: cudaMallocAsync(workspace)");
+    d_workspace = own;
+  } else if (ws_bytes < need) {
+    set_error("sg_evaluate_plane: workspace too small (%zu < %zu)", ws_bytes, need);
+    return SG_ERR_ARG;
+  }
+  sg_status st = launch_plane(g, d_alpha, origin, du, dv, width, height, d_image, dt, order, d_workspace, s);
+  if (own) cudaFreeAsync(own, s);
+  return st;
+}
+
 sg_status sg_evaluate_host(sg_grid g, const void* d_alpha, const void* h_x, uint64_t m, void* h_y, sg_dtype dt,
                            uint32_t flags, void* stream) {
   SG_CHECK_GRID(g);

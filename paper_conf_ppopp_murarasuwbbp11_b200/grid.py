@@ -98,6 +98,19 @@ class Grid:
         _sg.sg_evaluate_ordered(self._h, alpha, x.contiguous(), perm, first, count, y)
         return y
 
+    # ---- visualization slice (NEXT-3)
+    def render_plane(self, alpha: torch.Tensor, origin, du, dv, width: int, height: int, order: int = 1,
+                     out: torch.Tensor | None = None, workspace: torch.Tensor | None = None) -> torch.Tensor:
+        """(height, width) image of f_s at origin + (a+1/2) du + (b+1/2) dv (sg_evaluate_plane)."""
+        if alpha.numel() != self.num_points:
+            raise ValueError(f"alpha has {alpha.numel()} entries, the grid {self.num_points} points")
+        for v in (origin, du, dv):
+            if len(v) != self.d:
+                raise ValueError(f"origin, du, dv need {self.d} entries")
+        img = out if out is not None else torch.empty((height, width), dtype=alpha.dtype, device=alpha.device)
+        _sg.sg_evaluate_plane(self._h, alpha, origin, du, dv, img, order, workspace)
+        return img
+
     def evaluate_host(self, alpha: torch.Tensor, x_host, y_host=None, presorted: bool = False):
         if y_host is None:
             y_host = torch.empty(x_host.shape[0], dtype=x_host.dtype, pin_memory=True)

@@ -220,3 +220,36 @@ def test_gloo_world2_evaluate_distributed_on_one_gpu(tmp_path):
         assembled[own] = y[own]
     assert sorted(np.concatenate(owned).tolist()) == list(range(ref.size))
     assert np.array_equal(assembled, ref)
+
+
+# ----------------------------------------------------------------- visualization slice (NEXT-3)
+def plane_points(d, w, h, o, u, v, dtype):
+    a = np.arange(w, dtype=np.float64) + 0.5
+    b = np.arange(h, dtype=np.float64) + 0.5
+    x = (o[None, None, :] + a[None, :, None] * u[None, None, :]) + b[:, None, None] * v[None, None, :]
+    return x.reshape(h * w, d).astype(dtype)
+
+
+@pytest.mark.parametrize("d,n,dt,w,h", [(3, 14, "f32", 256, 128), (3, 8, "f64", 64, 36), (5, 6, "f64", 40, 20),
+                                        (10, 5, "f64", 33, 7), (2, 9, "f32", 16, 8)])
+def test_render_plane_equals_evaluate(P, torch, oracle, d, n, dt, w, h):
+    """sg_evaluate_plane: every pixel bitwise equal to sg_evaluate at the same point (row-major and
+    Morton-tiled visiting orders), and a sample of pixels against the oracle."""
+    g = P.Grid(d, n)
+    alpha = surpluses(torch, g, "A", dt, 0)
+    rng = np.random.default_rng(d * 100 + n)
+    if d == 3 and n == 14:  # the cfg4 plane (reading G19), scaled down
+        o, u, v = np.array([0.0, 0.0, 0.3]), np.array([1.0 / w, 0.0, 0.0]), np.array([0.0, 1.0 / h, 0.0])
+    else:  # an oblique slice, partly outside the cube
+        o = rng.random(d) * 0.3
+        u = (rng.random(d) - 0.3) / w
+        v = (rng.random(d) - 0.3) / h
+    npdt = np.float32 if dt == "f32" else np.float64
+    pts = torch.from_numpy(plane_points(d, w, h, o, u, v, npdt)).cuda()
+    ref = g.evaluate(alpha, pts, presorted=True).reshape(h, w)
+    for order in (0, 1):
+        img = g.render_plane(alpha, o, u, v, w, h, order=order)
+        assert torch.equal(img, ref), f"order {order}"
+    k = np.linspace(0, w * h - 1, 200).astype(np.int64)
+    yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy().astype(np.float64), pts.cpu().numpy()[k].astype(np.float64))
+    check_eval(ref.reshape(-1).cpu().numpy()[k], yo, ao, TOL[dt], f"plane d={d} n={n}")
