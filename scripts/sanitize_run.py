@@ -31,7 +31,7 @@ def run(d, n, dt=torch.float64, m=700, generic=False):
     if generic:
         _sg.sg_evaluate(g.handle, a, x, y, flags=_sg.SG_EVAL_GENERIC)
     perm = g.sfc_order(x)
-    g.evaluate_ordered(a, x, perm, 100, 300, out=y)
+    g.evaluate_ordered(a, x, perm, m // 7, m // 3, out=y)
     idx = torch.arange(min(g.num_points, 4096), dtype=torch.int64, device="cuda")
     l, i = g.idx2gp(idx)
     g.gp2idx(l, i)
