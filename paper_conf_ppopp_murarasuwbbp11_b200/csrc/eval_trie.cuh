@@ -72,6 +72,12 @@ struct Knobs {
   // inner (block) dimensions: blocks over dimensions 0..INNER-1 (smaller blocks and per-block register
   // arrays with INNER = 3; dimension 3 then becomes the innermost trie loop)
   static constexpr int INNER = 4;
+  // the block table C'[s] from a per-query, per-group table C_J[u] (u = s + sigma, compile-time index)
+  // computed once per group, instead of R+1 shift/logic pairs per block
+  static constexpr bool CST = false;
+  // RMIN prunes trie nodes (sub-tries of level sum < RMIN) but does not filter blocks: the complement of
+  // a launch with a larger INNER and RMAX = RMIN - 1 (whose blocks are exactly those sub-tries)
+  static constexpr bool RMIN_NODES_ONLY = false;
 };
 struct KnobsS0 : Knobs {
   static constexpr bool S0 = true;
@@ -83,9 +89,10 @@ struct Trie {
   static constexpr int O = D - I;          // outer (trie) dimensions
   static constexpr bool S0 = KN::S0, GO = KN::GO, LZ3 = KN::LZ3, H23 = KN::H23 && D >= 4;
   static constexpr bool D01 = KN::D01 && D >= 2;
+  static constexpr bool CST = KN::CST;
   // shared memory, [row][lane]: hat values of dimensions 2, 3 (read per block / slab), of
   // dimension I (per dimension-I node), then x of dimensions I+1..D-1
-  static constexpr int SM_IN = 2 * NM;
+  static constexpr int SM_IN = (I > 2 ? I - 2 : 0) * NM;  // hat rows of dimensions 2 .. I-1
   static constexpr int SM_PH = O > 0 ? NM : 0;
   static constexpr int SM_X = O > 1 ? O - 1 : 0;
   static constexpr int xrow(int t) { return t - I - 1; }
@@ -112,6 +119,7 @@ struct Trie {
     const T* rho;  // S0: this lane's column of the signed level-1/level-0 hat ratios
     T ph[I < 2 ? I : 2][D01 ? 1 : PHN];  // hat values of dimensions 0, 1 (registers), levels < PHN
     T d01[D01 ? PHN * (PHN + 1) / 2 : 1];  // D01: phi_0(r - l1) phi_1(l1) at index r (r + 1) / 2 + l1
+    uint32_t ct[CST ? NM : 1];             // CST: C_J[u] = (k_0 digits of level J above bit u) | (K_1 >> (NM-1-u))
     T ph23[H23 ? 2 : 1][H23 ? PHN : 1];  // H23: hat values of dimensions 2, 3 (registers)
     uint32_t K[D];
     double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
@@ -133,7 +141,7 @@ struct Trie {
   template <int J, int R>
   static __device__ __forceinline__ void block(Ctx& c, uint32_t P, T prod) {
     constexpr int NI = I;
-    if constexpr (R < RMIN || R > RMAX) {  // another launch evaluates this block
+    if constexpr ((R < RMIN && !KN::RMIN_NODES_ONLY) || R > RMAX) {  // another launch evaluates this block
       c.b += cnt(R, NI) << J;
       return;
     } else {
@@ -172,9 +180,13 @@ struct Trie {
     uint32_t Cs[R + 1];
 #pragma unroll
     for (int s = 0; s <= R; ++s) {
-      const uint32_t hi = K0J & ~((1u << (s + SG)) - 1u);
-      const uint32_t lo = (NI > 1) ? (k1 >> (NM - 1 - s - SG)) : 0u;
-      Cs[s] = hi | lo;
+      if constexpr (CST) {
+        Cs[s] = c.ct[CST ? s + SG : 0];
+      } else {
+        const uint32_t hi = K0J & ~((1u << (s + SG)) - 1u);
+        const uint32_t lo = (NI > 1) ? (k1 >> (NM - 1 - s - SG)) : 0u;
+        Cs[s] = hi | lo;
+      }
     }
     // hat values of dimensions 2, 3 for levels 0..R, from shared memory
     T ph2[R + 1], ph3[LZ3 ? 1 : R + 1];
@@ -188,50 +200,67 @@ struct Trie {
         if constexpr (!LZ3) ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
       }
     }
+    // INNER = 5: hat values of dimension 4 for levels 0..R, from shared memory
+    T ph4[NI >= 5 ? R + 1 : 1];
+    uint32_t k4 = 0;
+    if constexpr (NI >= 5) {
+#pragma unroll
+      for (int l = 0; l <= R; ++l) ph4[l] = phs_at(c.phs, 2 * NM + l);
+      asm volatile("mov.b32 %0, %1;" : "=r"(k4) : "r"(c.K[NI > 4 ? 4 : 0]));
+    }
     T acc = T(0);
-    constexpr int R3 = (NI >= 4) ? R : 0;
+    constexpr int R4 = (NI >= 5) ? R : 0;
     int cidx = 0;  // compile-time after unrolling: rank of the term inside the block
 #pragma unroll
-    for (int l3 = 0; l3 <= R3; ++l3) {
-      // k_3(l3) << SG
-      const uint32_t X3 = (NI >= 4) ? ((k3 >> (NM - 1 - l3 - SG)) & ~((1u << SG) - 1u)) : 0u;
-      const int R2 = (NI >= 3) ? R - l3 : 0;
-      T acc3 = T(0);
+    for (int l4 = 0; l4 <= R4; ++l4) {
+      // k_4(l4) << SG (INNER = 5); the dimensions <= 3 sit above bit SG4
+      const int SG4 = SG + l4;
+      const uint32_t X4 = (NI >= 5) ? ((k4 >> (NM - 1 - l4 - SG)) & ~((1u << SG) - 1u)) : 0u;
+      const int R3 = (NI >= 4) ? R - l4 : 0;
+      T acc4 = T(0);
 #pragma unroll
-      for (int l2 = 0; l2 <= R2; ++l2) {
-        // X_row = (k_2(l2) << (l3+SG)) | X3
-        uint32_t Xr = (NI >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG)) & ~((1u << (l3 + SG)) - 1u)) | X3) : X3;
-        asm("mov.b32 %0, %0;" : "+r"(Xr));
-        const uint32_t M = 0xffffffffu << (l2 + l3 + SG);
-        const int R1 = (NI >= 2) ? R - l3 - l2 : 0;
-        T acc2 = T(0);
+      for (int l3 = 0; l3 <= R3; ++l3) {
+        // k_3(l3) << SG4
+        const uint32_t X3 = (NI >= 4) ? (((k3 >> (NM - 1 - l3 - SG4)) & ~((1u << SG4) - 1u)) | X4) : X4;
+        const int R2 = (NI >= 3) ? R - l4 - l3 : 0;
+        T acc3 = T(0);
 #pragma unroll
-        for (int l1 = 0; l1 <= R1; ++l1) {
-          const int s = l1 + l2 + l3;
-          const int l0 = R - s;
-          uint32_t V;  // index1 - P = (C'[s] & M_row) | X_row: one LOP3
-          asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
-          const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
-          asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
-          const T a = __ldg(p + ((uint32_t)cidx << J));
-          if constexpr (D01) {
-            const int r = R - l2 - l3;
-            acc2 = fma(a, c.d01[D01 ? r * (r + 1) / 2 + l1 : 0], acc2);
-          } else if (NI >= 2) {
-            acc2 = fma(a * c.ph[0][D01 ? 0 : l0], c.ph[NI > 1 ? 1 : 0][D01 ? 0 : l1], acc2);
-          } else {
-            acc2 = fma(a, c.ph[0][D01 ? 0 : l0], acc2);
+        for (int l2 = 0; l2 <= R2; ++l2) {
+          // X_row = (k_2(l2) << (l3+SG4)) | X3
+          uint32_t Xr = (NI >= 3) ? (((k2 >> (NM - 1 - l2 - l3 - SG4)) & ~((1u << (l3 + SG4)) - 1u)) | X3) : X3;
+          asm("mov.b32 %0, %0;" : "+r"(Xr));
+          const uint32_t M = 0xffffffffu << (l2 + l3 + SG4);
+          const int R1 = (NI >= 2) ? R - l4 - l3 - l2 : 0;
+          T acc2 = T(0);
+#pragma unroll
+          for (int l1 = 0; l1 <= R1; ++l1) {
+            const int s = l1 + l2 + l3 + l4;
+            const int l0 = R - s;
+            uint32_t V;  // index1 - P = (C'[s] & M_row) | X_row: one LOP3
+            asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(V) : "r"(Cs[s]), "r"(M), "r"(Xr));
+            const T* p;  // &alpha[b + P + V] (one LEA pair); the term's c * 2^J is the load's immediate
+            asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(V), "n"((int)sizeof(T)), "l"(base));
+            const T a = __ldg(p + ((uint32_t)cidx << J));
+            if constexpr (D01) {
+              const int r = R - l2 - l3 - l4;
+              acc2 = fma(a, c.d01[D01 ? r * (r + 1) / 2 + l1 : 0], acc2);
+            } else if (NI >= 2) {
+              acc2 = fma(a * c.ph[0][D01 ? 0 : l0], c.ph[NI > 1 ? 1 : 0][D01 ? 0 : l1], acc2);
+            } else {
+              acc2 = fma(a, c.ph[0][D01 ? 0 : l0], acc2);
+            }
+            ++cidx;
           }
-          ++cidx;
+          acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
         }
-        acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
+        if constexpr (NI >= 4) {
+          const T h3 = LZ3 ? phs_at(c.phs, 1 * NM + l3) : ph3[LZ3 ? 0 : l3];
+          acc4 = fma(acc3, h3, acc4);
+        } else {
+          acc4 = acc3;
+        }
       }
-      if constexpr (NI >= 4) {
-        const T h3 = LZ3 ? phs_at(c.phs, 1 * NM + l3) : ph3[LZ3 ? 0 : l3];
-        acc = fma(acc3, h3, acc);
-      } else {
-        acc = acc3;
-      }
+      acc = (NI >= 5) ? fma(acc4, ph4[NI >= 5 ? l4 : 0], acc) : acc4;
     }
     c.res = fma((double)acc, (double)prod, c.res);
     c.b += cnt(R, NI) << J;
@@ -407,6 +436,12 @@ struct Trie {
   static __device__ __forceinline__ void groups(Ctx& c, int n) {
     if constexpr (J <= J1 && J < NM) {
       if (J < n) {
+        if constexpr (CST) {
+          const uint32_t K0J = c.K[0] >> (NM - 1 - J);
+#pragma unroll
+          for (int u = 0; u <= J; ++u)
+            c.ct[CST ? u : 0] = (K0J & ~((1u << u) - 1u)) | ((I > 1) ? (c.K[I > 1 ? 1 : 0] >> (NM - 1 - u)) : 0u);
+        }
         if constexpr (O == 0) block<J, J>(c, 0u, T(1));  // no outer dimensions: one block per group
         else node<J, D - 1>(c, J, 0u, T(1));
         groups<J + 1, J1>(c, n);

@@ -82,13 +82,26 @@ static sg_status d10_split3(const Layout& L, const double* a, const double* x, c
   return st;
 }
 
-template <int RL, bool HH, int TL, bool DD = false>
+template <int RL, bool HH, int TL, bool DD = false, bool CT = false>
 struct KLowX : trie::Knobs {
   static constexpr int RMAX = RL;
   static constexpr bool H23 = HH;
   static constexpr int TAIL = TL;
   static constexpr bool D01 = DD;
+  static constexpr bool CST = CT;
 };
+template <bool DD, bool CT>
+static sg_status d10_splitc(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                            double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLowX<6, false, 3, false, CT>>(L, a, x, p, m, y, s);
+#define SG_R(J)                                                                                                        \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, J, J, KLowX<4, false, 3, DD, CT>>(L, a, x, p, m, y, s); \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, J, J, KHigh<4>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
 template <int RL>
 static sg_status d10_splitd(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
                             double* y, cudaStream_t s) {
@@ -152,6 +165,35 @@ static sg_status d10_splith(const Layout& L, const double* a, const double* x, c
   return st;
 }
 
+// INNER = 5 for the small-block launch: blocks = sub-tries of dimensions 0..4 with level sum <= RL;
+// the large-block launch (INNER = 4) prunes exactly those sub-tries (node budget at dimension 4 <= RL)
+template <int RL>
+struct KLow5 : trie::Knobs {
+  static constexpr int RMAX = RL;
+  static constexpr int INNER = 5;
+};
+template <int RL>
+struct KHighN : trie::Knobs {
+  static constexpr int RMIN = RL + 1;
+  static constexpr bool RMIN_NODES_ONLY = true;
+};
+template <int RL, bool I5LOW06>
+static sg_status d10_split5(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m,
+                            double* y, cudaStream_t s) {
+  sg_status st = SG_OK;
+  if constexpr (I5LOW06) {
+    if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLow5<6>>(L, a, x, p, m, y, s);
+  } else {
+    if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLow<6>>(L, a, x, p, m, y, s);
+  }
+#define SG_R(J)                                                                                          \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, J, J, KLow5<RL>>(L, a, x, p, m, y, s);  \
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, J, J, KHighN<RL>>(L, a, x, p, m, y, s);
+  SG_R(7) SG_R(8) SG_R(9) SG_R(10)
+#undef SG_R
+  return st;
+}
+
 // returns true if an experiment variant handled the call
 bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint32_t* perm, uint64_t m, void* y,
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
@@ -172,10 +214,11 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "GO4")) { *st = d10_go<4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SPLIT4B")) { *st = d10_split<4, 4, 4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SD4")) { *st = d10_splitd<4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SD3")) { *st = d10_splitd<3>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SH33")) { *st = d10_splith<3, false>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SH34")) { *st = d10_splith<4, false>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SH34D")) { *st = d10_splith<4, true>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SC")) { *st = d10_splitc<false, true>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SCD")) { *st = d10_splitc<true, true>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S5A4")) { *st = d10_split5<4, false>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S5A5")) { *st = d10_split5<5, false>(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "S5B4")) { *st = d10_split5<4, true>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SXT")) { *st = d10_splitx<false, 4>(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
