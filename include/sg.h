@@ -184,6 +184,20 @@ sg_status sg_evaluate_plane(sg_grid g, const void *d_alpha, const double *origin
                             uint32_t width, uint32_t height, void *d_image, sg_dtype dt, uint32_t order,
                             void *d_workspace, size_t ws_bytes, void *stream);
 
+/* Grids sharded across devices (the paper's evaluation is a sum over subspaces,
+ * Alg. 7, so it splits into partial sums over disjoint subspace sets).  The layout is cut
+ * into `parts` contiguous index ranges at (level group j, level l_{d-1}) boundaries -- whole groups for
+ * d <= 5 -- each holding about 1/parts of the subspaces, i.e. of the evaluation work.
+ * sg_part_bounds: the range [*first, *first + *count) of part `part` (host only, any grid).
+ * sg_evaluate_part: d_y[q] (+)= the part's share of f_s(x_q), q < m (accumulate != 0 adds to d_y),
+ * with d_alpha_part holding ONLY the part's *count surpluses (alpha[first .. first+count)); summing the
+ * parts' results (e.g. one NCCL all-reduce) gives f_s up to rounding.  d_perm (may be NULL) orders the
+ * queries as in sg_evaluate_ordered.  Generic kernels only: d <= 12, n <= 12, N < 2^32 (SG_ERR_ARG
+ * otherwise).  Asynchronous. */
+sg_status sg_part_bounds(sg_grid g, uint32_t parts, uint32_t part, uint64_t *first, uint64_t *count);
+sg_status sg_evaluate_part(sg_grid g, const void *d_alpha_part, uint32_t parts, uint32_t part, const void *d_x,
+                           uint64_t m, const uint32_t *d_perm, void *d_y, int accumulate, sg_dtype dt, void *stream);
+
 /* End-to-end evaluation from HOST buffers: copies h_x (m x d) to the device,
  * evaluates as sg_evaluate, copies the m results to h_y.  d_alpha is on the
  * device.  Device buffers are allocated stream-ordered.  The three steps run

@@ -56,6 +56,8 @@ _SIGS = {
     "sg_sfc_order": [_p, _p, _u64, ctypes.c_int, _p, _p, _sz, _p],
     "sg_evaluate_ordered": [_p, _p, _p, _u64, _p, _u64, _u64, _p, ctypes.c_int, _p],
     "sg_plane_workspace_bytes": [_p, _u32, _u32, ctypes.c_int, ctypes.POINTER(_sz)],
+    "sg_part_bounds": [_p, _u32, _u32, ctypes.POINTER(_u64), ctypes.POINTER(_u64)],
+    "sg_evaluate_part": [_p, _p, _u32, _u32, _p, _u64, _p, _p, ctypes.c_int, ctypes.c_int, _p],
     "sg_evaluate_plane": [_p, _p, _p, _p, _p, _u32, _u32, _p, ctypes.c_int, _u32, _p, _sz, _p],
 }
 for _name, _args in _SIGS.items():
@@ -247,6 +249,21 @@ def sg_evaluate_plane(g, alpha: torch.Tensor, origin, du, dv, image: torch.Tenso
     _check(lib.sg_evaluate_plane(g, _dev(alpha, "alpha"), _np_ptr(o), _np_ptr(u), _np_ptr(v), w, h,
                                  _dev(image, "image"), _dtype_code(alpha), order, ws, wsb, _stream(stream)),
            "sg_evaluate_plane")
+
+
+def sg_part_bounds(g, parts: int, part: int) -> tuple[int, int]:
+    first, count = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib.sg_part_bounds(g, parts, part, ctypes.byref(first), ctypes.byref(count)), "sg_part_bounds")
+    return int(first.value), int(count.value)
+
+
+def sg_evaluate_part(g, alpha_part: torch.Tensor, parts: int, part: int, x: torch.Tensor, y: torch.Tensor,
+                     perm: torch.Tensor | None = None, accumulate: bool = False, stream=None) -> None:
+    _check_batch(alpha_part, x, y)
+    pp = _dev(perm, "perm") if perm is not None else None
+    ap = _dev(alpha_part, "alpha_part") if alpha_part.numel() else None
+    _check(lib.sg_evaluate_part(g, ap, parts, part, _dev(x, "x"), x.shape[0], pp, _dev(y, "y"), 1 if accumulate else 0,
+                                _dtype_code(x), _stream(stream)), "sg_evaluate_part")
 
 
 def sg_evaluate_host(g, alpha: torch.Tensor, x_host, y_host, flags: int = 0, stream=None) -> None:

@@ -81,6 +81,13 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
 sg_status launch_evaluate(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                           void* y, sg_dtype dt, uint32_t flags, cudaStream_t s);
 size_t plane_workspace_bytes(int d, uint64_t m, size_t elem);
+// a part of the subspaces for the generic kernel (sharded grids): groups j0..j1, l_{d-1} from v0 in group
+// j0 to v1 in group j1, running base starting at b0; accumulate adds to y
+struct GenPart {
+  int j0 = 0, v0 = 0, j1 = 64, v1 = 64;
+  uint32_t b0 = 0;
+  int accumulate = 0;
+};
 sg_status launch_plane(const sg_grid_s* g, const void* alpha, const double* origin, const double* du, const double* dv,
                        uint32_t width, uint32_t height, void* img, sg_dtype dt, uint32_t order, void* ws,
                        cudaStream_t s);

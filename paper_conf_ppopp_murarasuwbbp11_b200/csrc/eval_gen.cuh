@@ -45,6 +45,7 @@ struct GTrie {
     double res;
     uint32_t b;  // running subspace base (elements), warp-uniform
     int J;       // current level group (run time)
+    int vlo, vhi;  // levels l_{D-1} of the top trie loop this launch evaluates (a part of a sharded grid)
   };
 
   static constexpr uint32_t cnt(int R) {  // subspaces per block = C(R+I-1, I-1)
@@ -166,7 +167,13 @@ struct GTrie {
       inner_tail<kTail>(c, B, P, prod);
     } else {
       T u = c.xs[xrow(t) * NT];
-      for (int lt = 0; lt <= B; ++lt) {
+      int lt0 = 0, lt1 = B;
+      if (t == D - 1) {  // the top loop: a part of a sharded grid may start / end inside it
+        lt0 = c.vlo;
+        lt1 = c.vhi < B ? c.vhi : B;
+        for (int k = 0; k < lt0; ++k) u = dbl_u(u);
+      }
+      for (int lt = lt0; lt <= lt1; ++lt) {
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
         node<t - 1>(c, B - lt, P | (kt << SG), prod * hat_u(u));
         u = dbl_u(u);
@@ -178,7 +185,7 @@ struct GTrie {
 template <typename T, int D, int NT, int MINB>
 __global__ void __launch_bounds__(NT, MINB)
     k_eval_gen(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
-               int n, T* __restrict__ y) {
+               int n, T* __restrict__ y, int j0, int v0, int j1, int v1, uint32_t b0, int accumulate) {
   using TR = GTrie<T, D, NT>;
   constexpr int I = TR::I, NM = TR::NM;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -215,17 +222,28 @@ __global__ void __launch_bounds__(NT, MINB)
     }
   }
   c.res = 0.0;
-  c.b = 0;
-  for (int J = 0; J < n; ++J) {  // level groups in the bijection order
+  c.b = b0;  // index3(j0) + the subspaces of group j0 before level l_{D-1} = v0 (times 2^j0)
+  // level groups in the bijection order; a sharded grid's part (sg_evaluate_part) covers
+  // the groups j0..j1, starting at l_{D-1} = v0 in group j0 and ending at l_{D-1} = v1 in group j1
+  for (int J = j0; J <= j1 && J < n; ++J) {
     c.J = J;
+    c.vlo = J == j0 ? v0 : 0;
+    c.vhi = J == j1 ? v1 : J;
     if constexpr (TR::O == 0) TR::leaf(c, J, 0u, T(1));  // one block per group
     else TR::template node<D - 1>(c, J, 0u, T(1));
   }
-  if (active) y[src] = bad ? T(NAN) : (T)c.res;
+  if (active) {
+    double r = c.res;
+    if (accumulate) r += (double)y[src];
+    y[src] = bad ? T(NAN) : (T)r;
+  }
 }
 
+// Part of the groups: j0..j1 with l_{D-1} in [v0, ..] in group j0 and [.., v1] in group j1 (D >= 6; whole groups
+// otherwise), the running base starting at b0; accumulate adds to y.  Default: the whole grid.
 template <typename T, int D>
-sg_status launch_gen(const T* alpha, const T* x, const uint32_t* perm, uint64_t m, int n, T* y, cudaStream_t s) {
+sg_status launch_gen(const T* alpha, const T* x, const uint32_t* perm, uint64_t m, int n, T* y, cudaStream_t s,
+                     int j0 = 0, int v0 = 0, int j1 = 64, int v1 = 64, uint32_t b0 = 0, int accumulate = 0) {
   constexpr int NT = 128, MINB = 3;
   using TR = GTrie<T, D, NT>;
   auto kern = k_eval_gen<T, D, NT, MINB>;
@@ -235,7 +253,7 @@ sg_status launch_gen(const T* alpha, const T* x, const uint32_t* perm, uint64_t 
   const sg_status st = set_smem_attr(kern, attr_done, smem, pct, "cudaFuncSetAttribute(k_eval_gen)");
   if (st != SG_OK) return st;
   const unsigned blocks = (unsigned)((m + NT - 1) / NT);
-  kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, n, y);
+  kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, n, y, j0, v0, j1, v1, b0, accumulate);
   return launched("k_eval_gen");
 }
 

@@ -1,22 +1,29 @@
 // eval_trie_d10a.cu -- instantiations of the evaluation kernel (eval_trie.cuh) for d = 10, n <= 11 (cfg3),
 // groups 0..8.  One launch per (level-group range, block-budget range); consecutive launches accumulate
-// into y.  Groups >= 7 are split by block budget R: the launch of the many small blocks (R <= 4, ~60%
-// of the terms) holds the register hat tables of dimensions 0, 1 only up to level 4 and runs 16
-// warps/SM (128 registers, no spills); the launch of the large blocks (R >= 5) keeps 12 warps/SM and
-// prunes every sub-trie of budget < 5.  Measured +8% over one launch per group at 12 warps
-// (profiles/r02_split.txt).  Split across files only so that nvcc compiles them in parallel.
+// into y.  Groups >= 7 are split by budget: the small-block launch evaluates the sub-tries of dimensions
+// 0..4 whose level sum is <= 4 as blocks of 5 inner dimensions (INNER = 5: C(R+4, 4) consecutive
+// subspaces per block) with the register hat tables of dimensions 0, 1 only up to level 4, at 16
+// warps/SM (128 registers); the large-block launch (blocks over dimensions 0..3, 12 warps/SM) prunes
+// exactly those sub-tries.  Groups 0-6 run as small blocks (R <= 6) at 16 warps/SM.  Measured +8% (split
+// at 4 dimensions) and +3% more (5 inner dimensions for the small blocks) over one launch per group at 12
+// warps/SM (profiles/r02_split.txt).  Split across files only so that nvcc compiles them in parallel.
 #include "eval_trie.cuh"
 
 namespace sg {
 
 namespace d10 {
+// small blocks: sub-tries of dimensions 0..4 (INNER = 5) with level sum <= RL
 template <int RL>
 struct KLow : trie::Knobs {
   static constexpr int RMAX = RL;
+  static constexpr int INNER = 5;
 };
+// large blocks: blocks over dimensions 0..3 of every dimension-4 node with budget > RL (exactly the
+// complement: the nodes of budget <= RL are the small-block launch's blocks)
 template <int RL>
 struct KHigh : trie::Knobs {
   static constexpr int RMIN = RL + 1;
+  static constexpr bool RMIN_NODES_ONLY = true;
 };
 }  // namespace d10
 

@@ -6,13 +6,18 @@
 namespace sg {
 
 namespace d10b {
+// small blocks: sub-tries of dimensions 0..4 (INNER = 5) with level sum <= RL
 template <int RL>
 struct KLow : trie::Knobs {
   static constexpr int RMAX = RL;
+  static constexpr int INNER = 5;
 };
+// large blocks: blocks over dimensions 0..3 of every dimension-4 node with budget > RL (exactly the
+// complement: the nodes of budget <= RL are the small-block launch's blocks)
 template <int RL>
 struct KHigh : trie::Knobs {
   static constexpr int RMIN = RL + 1;
+  static constexpr bool RMIN_NODES_ONLY = true;
 };
 }  // namespace d10b
 

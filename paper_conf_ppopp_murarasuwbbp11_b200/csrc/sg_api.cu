@@ -80,21 +80,82 @@ sg_status launch_eval_simple(const sg_grid_s* g, const void* alpha, const void* 
                              void* y, sg_dtype dt, cudaStream_t s);
 #define SG_GEN_DECL(part)                                                                                      \
   bool launch_gen_##part(int d, int n, bool f64, const void* a, const void* x, const uint32_t* p, uint64_t m, \
-                         void* y, cudaStream_t s, sg_status* st);
+                         void* y, cudaStream_t s, sg_status* st, const GenPart& pt);
 SG_GEN_DECL(a) SG_GEN_DECL(b) SG_GEN_DECL(c) SG_GEN_DECL(d)
 #undef SG_GEN_DECL
 
 // the generic run-time-level kernel (eval_gen.cuh): d <= 12, n <= 12; 32-bit offsets
 static sg_status launch_eval_gen(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm,
-                                 uint64_t m, void* y, sg_dtype dt, cudaStream_t s, bool* handled) {
+                                 uint64_t m, void* y, sg_dtype dt, cudaStream_t s, bool* handled,
+                                 const GenPart& pt = GenPart()) {
   *handled = false;
   const int d = g->L.d, n = g->L.n;
-  if (n > 12 || m > 0xffffffffull || g->L.N >= 0xffffffffull) return SG_OK;
+  if (n > 12 || d > 12 || m > 0xffffffffull || g->L.N >= 0xffffffffull) return SG_OK;
   sg_status st = SG_OK;
   const bool f64 = dt == SG_F64;
-  *handled = launch_gen_a(d, n, f64, alpha, x, perm, m, y, s, &st) || launch_gen_b(d, n, f64, alpha, x, perm, m, y, s, &st) ||
-             launch_gen_c(d, n, f64, alpha, x, perm, m, y, s, &st) || launch_gen_d(d, n, f64, alpha, x, perm, m, y, s, &st);
+  *handled = launch_gen_a(d, n, f64, alpha, x, perm, m, y, s, &st, pt) ||
+             launch_gen_b(d, n, f64, alpha, x, perm, m, y, s, &st, pt) ||
+             launch_gen_c(d, n, f64, alpha, x, perm, m, y, s, &st, pt) ||
+             launch_gen_d(d, n, f64, alpha, x, perm, m, y, s, &st, pt);
   return st;
+}
+
+// ---- sharded grids: the layout cut into contiguous parts at (group j, level l_{d-1} = v)
+// unit boundaries (whole groups for d <= 5, whose generic kernel has no separate top trie loop), each part
+// holding about 1/parts of the subspaces (= of the evaluation work: one gather per subspace per query).
+struct PartRange {
+  GenPart gp;
+  uint64_t first, count;
+};
+static void part_range(const Layout& L, uint32_t parts, uint32_t part, PartRange* out) {
+  const int d = L.d, n = L.n;
+  const bool fine = d >= 6;
+  struct Unit {
+    int j, v;
+    uint64_t subs;
+  };
+  std::vector<Unit> units;  // in layout order: group j ascending, then l_{d-1} ascending (Alg. 3: slowest)
+  for (int j = 0; j < n; ++j) {
+    if (!fine) {
+      units.push_back({j, -1, L.cnt[j]});
+      continue;
+    }
+    for (int v = 0; v <= j; ++v) units.push_back({j, v, L.C(d - 2, j - v)});  // C(j-v+d-2, d-2) subspaces
+  }
+  // part p takes the units whose cumulative start lies in [p T / parts, (p+1) T / parts)
+  const uint64_t lo = (uint64_t)((unsigned __int128)L.T * part / parts);
+  const uint64_t hi = (uint64_t)((unsigned __int128)L.T * (part + 1) / parts);
+  uint64_t cum = 0;
+  int ua = -1, ub = -1;
+  for (size_t u = 0; u < units.size(); ++u) {
+    if (cum >= lo && cum < hi) {
+      if (ua < 0) ua = (int)u;
+      ub = (int)u;
+    }
+    cum += units[u].subs;
+  }
+  out->gp = GenPart();
+  if (ua < 0) {  // empty part (more parts than units)
+    out->gp.j0 = 1;
+    out->gp.j1 = 0;
+    out->first = out->count = 0;
+    return;
+  }
+  auto unit_first = [&](int u) {  // index3(j) + (subspaces of group j before the unit) 2^j
+    const int j = units[u].j;
+    uint64_t before = 0;
+    for (int w = u - 1; w >= 0 && units[w].j == j; --w) before += units[w].subs;
+    return L.off[j] + (before << j);
+  };
+  const uint64_t first = unit_first(ua);
+  const uint64_t last = unit_first(ub) + (units[ub].subs << units[ub].j);
+  out->gp.j0 = units[ua].j;
+  out->gp.v0 = fine ? units[ua].v : 0;
+  out->gp.j1 = units[ub].j;
+  out->gp.v1 = fine ? units[ub].v : 64;
+  out->gp.b0 = (uint32_t)first;
+  out->first = first;
+  out->count = last - first;
 }
 sg_status launch_eval_trie(const sg_grid_s* g, const void* alpha, const void* x, const uint32_t* perm, uint64_t m,
                            void* y, sg_dtype dt, cudaStream_t s, bool* handled);
@@ -431,6 +492,67 @@ sg_status sg_evaluate_plane(sg_grid g, const void* d_alpha, const double* origin
   }
   sg_status st = launch_plane(g, d_alpha, origin, du, dv, width, height, d_image, dt, order, d_workspace, s);
   if (own) cudaFreeAsync(own, s);
+  return st;
+}
+
+sg_status sg_part_bounds(sg_grid g, uint32_t parts, uint32_t part, uint64_t* first, uint64_t* count) {
+  SG_CHECK_GRID(g);
+  if (parts == 0 || part >= parts || !first || !count) {
+    set_error("sg_part_bounds: need 0 <= part < parts and non-NULL outputs");
+    return SG_ERR_ARG;
+  }
+  PartRange pr;
+  part_range(g->L, parts, part, &pr);
+  *first = pr.first;
+  *count = pr.count;
+  return SG_OK;
+}
+
+sg_status sg_evaluate_part(sg_grid g, const void* d_alpha_part, uint32_t parts, uint32_t part, const void* d_x,
+                           uint64_t m, const uint32_t* d_perm, void* d_y, int accumulate, sg_dtype dt, void* stream) {
+  SG_CHECK_GRID(g);
+  SG_CHECK_DEVICE(g);
+  if (!dtype_ok(dt)) return SG_ERR_DTYPE;
+  if (parts == 0 || part >= parts) {
+    set_error("sg_evaluate_part: need 0 <= part < parts");
+    return SG_ERR_ARG;
+  }
+  if (m == 0) return SG_OK;
+  if (!d_x || !d_y) {
+    set_error("sg_evaluate_part: NULL buffer");
+    return SG_ERR_ARG;
+  }
+  if (g->L.d > 12 || g->L.n > 12 || g->L.N >= 0xffffffffull || m > 0x7fffffffull) {
+    set_error("sg_evaluate_part: sharded evaluation needs d <= 12, n <= 12, N < 2^32, m < 2^31");
+    return SG_ERR_ARG;
+  }
+  PartRange pr;
+  part_range(g->L, parts, part, &pr);
+  DeviceGuard guard(g->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  if (pr.count == 0) {  // an empty part adds nothing; without accumulate y is defined as 0
+    if (!accumulate) {
+      cudaError_t e = cudaMemsetAsync(d_y, 0, m * dtype_size(dt), s);
+      if (e != cudaSuccess) return cuda_fail(e, "sg_evaluate_part: cudaMemsetAsync");
+    }
+    return SG_OK;
+  }
+  if (!d_alpha_part) {
+    set_error("sg_evaluate_part: NULL surpluses");
+    return SG_ERR_ARG;
+  }
+  GenPart gp = pr.gp;
+  gp.accumulate = accumulate ? 1 : 0;
+  // the kernel indexes the surpluses with global offsets: hand it the part's base shifted by its first
+  // index (only the part's own count values are ever read)
+  const void* base = (const char*)d_alpha_part - pr.first * dtype_size(dt);
+  ProfScope prof(kProfEval, s);
+  bool handled = false;
+  const sg_status st = launch_eval_gen(g, base, d_x, d_perm, m, d_y, dt, s, &handled, gp);
+  if (st == SG_OK && !handled) {
+    set_error("sg_evaluate_part: no generic kernel for d=%d", g->L.d);
+    return SG_ERR_ARG;
+  }
   return st;
 }
 

@@ -98,6 +98,22 @@ class Grid:
         _sg.sg_evaluate_ordered(self._h, alpha, x.contiguous(), perm, first, count, y)
         return y
 
+    # ---- sharded grids (NEXT-4)
+    def part_bounds(self, parts: int, part: int) -> tuple[int, int]:
+        """(first, count): part `part` of `parts` contiguous, work-balanced ranges of the layout."""
+        return _sg.sg_part_bounds(self._h, parts, part)
+
+    def evaluate_part(self, alpha_part: torch.Tensor, parts: int, part: int, x: torch.Tensor,
+                      out: torch.Tensor | None = None, perm: torch.Tensor | None = None,
+                      accumulate: bool = False) -> torch.Tensor:
+        """The part's share of f_s at every query (alpha_part = the part's surpluses only)."""
+        first, count = self.part_bounds(parts, part)
+        if alpha_part.numel() != count:
+            raise ValueError(f"part {part}/{parts} holds {count} surpluses, got {alpha_part.numel()}")
+        y = out if out is not None else torch.empty(x.shape[0], dtype=x.dtype, device=x.device)
+        _sg.sg_evaluate_part(self._h, alpha_part, parts, part, x.contiguous(), y, perm, accumulate)
+        return y
+
     # ---- visualization slice (NEXT-3)
     def render_plane(self, alpha: torch.Tensor, origin, du, dv, width: int, height: int, order: int = 1,
                      out: torch.Tensor | None = None, workspace: torch.Tensor | None = None) -> torch.Tensor:

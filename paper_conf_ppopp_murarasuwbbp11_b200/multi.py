@@ -60,6 +60,22 @@ def evaluate_distributed(grid, alpha, x, group=None, src: int = 0, out=None, per
     return y, perm, first, count
 
 
+def evaluate_sharded_grid(grid, alpha_part, x, group=None, out=None):
+    """Evaluate a grid whose surpluses are sharded across the ranks (grids larger than
+    one GPU): rank r holds only part r of P (``grid.part_bounds(P, r)``: a contiguous, work-balanced range of
+    the layout) and evaluates that part's share of f_s at EVERY query of the batch ``x``; one all-reduce
+    (sum) of the m results -- the path's only collective, m values instead of the N surpluses -- gives
+    every rank f_s(x).  Parts are summed in rank order by the collective, so the result equals one-GPU
+    evaluation up to rounding (not bitwise)."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    y = grid.evaluate_part(alpha_part, world, rank, x, out=out)
+    if world > 1:
+        dist.all_reduce(y, op=dist.ReduceOp.SUM, group=group)
+    return y
+
+
 def checksum(t) -> int:
     """Order-sensitive 64-bit checksum of a tensor's bytes (for replication checks)."""
     import numpy as np

@@ -253,3 +253,67 @@ def test_render_plane_equals_evaluate(P, torch, oracle, d, n, dt, w, h):
     k = np.linspace(0, w * h - 1, 200).astype(np.int64)
     yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy().astype(np.float64), pts.cpu().numpy()[k].astype(np.float64))
     check_eval(ref.reshape(-1).cpu().numpy()[k], yo, ao, TOL[dt], f"plane d={d} n={n}")
+
+
+# ----------------------------------------------------------------- sharded grids (NEXT-4)
+@pytest.mark.parametrize("d,n,parts", [(3, 7, 3), (6, 6, 4), (10, 8, 8), (10, 11, 2), (12, 5, 5), (7, 5, 40)])
+def test_evaluate_parts_sum_to_the_grid(P, torch, oracle, d, n, parts):
+    """The parts of sg_part_bounds tile the layout exactly (contiguous, in order); each part evaluated from
+    ONLY its own surpluses (a copy of its slice) sums to the whole-grid evaluation within the normwise
+    tolerance, and a sample agrees with the oracle."""
+    g = P.Grid(d, n)
+    alpha = surpluses(torch, g, "B", "f64", d + n)
+    m = 20_000 if g.num_points < 5e7 else 2_000
+    x = S.queries_torch(d, m, 31 * d + n, device="cuda")
+    bounds = [g.part_bounds(parts, r) for r in range(parts)]
+    pos = 0
+    for first, count in bounds:
+        assert first == pos or count == 0
+        pos = first + count if count else pos
+    assert pos == g.num_points
+    y = torch.zeros(m, dtype=torch.float64, device="cuda")
+    for r, (first, count) in enumerate(bounds):
+        part = alpha[first:first + count].clone()  # the part's surpluses only
+        g.evaluate_part(part, parts, r, x, out=y, accumulate=True)
+    ref = g.evaluate(alpha, x)
+    k = np.linspace(0, m - 1, 64).astype(np.int64)
+    yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy(), x.cpu().numpy()[k])
+    check_eval(y.cpu().numpy()[k], yo, ao, TOL["f64"], f"parts d={d} n={n} P={parts}")
+    # whole batch against the one-call result: normwise with the oracle's A(x) scale bound |y| <= A
+    err = (y - ref).abs().max().item()
+    assert err <= 1e-12 * float(np.max(ao)) * 10, err
+
+
+def _shard_worker(rank, world, port, outdir):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_murarasuwbbp11_b200 as P
+    from paper_conf_ppopp_murarasuwbbp11_b200 import multi
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        g = P.Grid(8, 7)
+        alpha = g.hierarchize_(S.f_A_torch(g.coords()))  # (every rank computes it here; it keeps only its part)
+        first, count = g.part_bounds(world, rank)
+        mine = alpha[first:first + count].clone()
+        del alpha
+        x = S.queries_torch(8, 30_001, 77, device="cuda")
+        y = multi.evaluate_sharded_grid(g, mine, x)  # own part + one all-reduce
+        torch.cuda.synchronize()
+        np.save(os.path.join(outdir, f"y{rank}.npy"), y.cpu().numpy())
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_sharded_grid_on_one_gpu(P, torch, tmp_path):
+    import torch.multiprocessing as mp
+    world = 2
+    mp.spawn(_shard_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    g = P.Grid(8, 7)
+    alpha = g.hierarchize_(S.f_A_torch(g.coords()))
+    ref = g.evaluate(alpha, S.queries_torch(8, 30_001, 77, device="cuda")).cpu().numpy()
+    y0, y1 = np.load(tmp_path / "y0.npy"), np.load(tmp_path / "y1.npy")
+    assert np.array_equal(y0, y1)  # every rank holds the reduced result
+    np.testing.assert_allclose(y0, ref, rtol=1e-12, atol=0)  # positive surpluses: plain relative error

@@ -146,3 +146,36 @@ def test_budget1_hat_ratio_reading():
     for xv in [0.25, 0.49999999, 0.5, 0.75, 1.0 - 2.0 ** -40]:
         k = int(np.clip(np.floor(2.0 * xv), 0, 1))
         assert k == (1 if xv >= 0.5 else 0)
+
+
+@pytest.mark.parametrize("d,n", [(1, 6), (3, 7), (5, 4), (6, 6), (10, 11), (12, 5)])
+def test_part_bounds_tile_the_layout(P, oracle, d, n):
+    """sg_part_bounds (sharded grids, NEXT-4): P parts are contiguous, in layout order, cover [0, N) exactly,
+    start at (group, l_{d-1}) boundaries (whole groups for d <= 5), and balance the subspace count."""
+    h, N = P.sg_create(d, n)
+    try:
+        for parts in (1, 2, 3, 8):
+            pos, subs = 0, []
+            for r in range(parts):
+                first, count = P.sg_part_bounds(h, parts, r)
+                if count == 0:
+                    subs.append(0)
+                    continue
+                assert first == pos
+                pos = first + count
+                # the part starts at a unit boundary: the point at `first` has its own subspace's first cell
+                # and (for d <= 5) level sum = a group start
+                l, i = oracle.idx2gp(d, n, np.array([first], dtype=np.uint64))
+                assert np.all(i == 1)
+                if d <= 5:
+                    assert first in [oracle.index3(d, j) for j in range(n)]
+                # subspaces in the part
+                ls, _ = oracle.idx2gp(d, n, np.arange(first, first + count, dtype=np.uint64))
+                subs.append(len({tuple(r_) for r_ in ls}) if count < 2_000_000 else None)
+            assert pos == N
+            T = oracle.binom(n - 1 + d, d)
+            if parts > 1 and all(s is not None for s in subs) and d >= 6:
+                unit = oracle.binom(n - 1 + d - 2, d - 2)  # the largest (group, l_{d-1}) unit
+                assert sum(subs) == T and max(subs) <= -(-T // parts) + unit
+    finally:
+        P.sg_destroy(h)
