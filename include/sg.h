@@ -198,6 +198,34 @@ sg_status sg_part_bounds(sg_grid g, uint32_t parts, uint32_t part, uint64_t *fir
 sg_status sg_evaluate_part(sg_grid g, const void *d_alpha_part, uint32_t parts, uint32_t part, const void *d_x,
                            uint64_t m, const uint32_t *d_perm, void *d_y, int accumulate, sg_dtype dt, void *stream);
 
+/* ---- Sparse grids with NON-ZERO boundary (Sec. 4.4, Fig. 7).
+ * "The boundary of a d-dimensional sparse grid is composed of lower-dimensional, zero-boundary sparse grids":
+ * the grid is the list of the 3^d FACES (S, c) -- S the free dimensions, c in {0,1}^{d-|S|} the values of
+ * the fixed ones -- each carrying the |S|-dimensional zero-boundary grid of level n (the interior is S = all,
+ * the corners |S| = 0: one point).  Layout (reading G20; the paper leaves the ordering function open):
+ * faces grouped by dimensionality |S| = d, d-1, ..., 0, inside a group by the free-dimension bitmask
+ * ascending, then by the fixed values as a binary number (bit k = value of the k-th fixed dimension);
+ * inside a face the |S|-dimensional layout above over the free dimensions in increasing order.
+ * Basis: phi_p(x) = prod_{t in S} phi_{l_t,i_t}(x_t) prod_{t not in S} b_{c_t}(x_t), b_0(x) = 1-x, b_1(x) = x
+ * on [0,1]; f_s = 0 outside [0,1]^d; NaN propagates.  1 <= d <= 12, 1 <= n <= 14.
+ * sg_bcreate/sg_bdestroy: the handle (host layout; device tables when a GPU is present).
+ * sg_bface: the layout of face `face` (< 3^d): free mask, fixed bits, first index, point count.
+ * sg_bcoords_device: the coordinates (N x d, layout order) of every point, exact.
+ * sg_bhierarchize: in place, nodal values -> surpluses, dimension by dimension (t = 0..d-1): every point of
+ *   a face with t free becomes v - (v_L + v_R)/2 with its 1D parents at x_t -+ 2^-(l_t+1) (on the face
+ *   fixing t to 0 / 1 when the parent coordinate is 0 / 1), values of pass t-1.
+ * sg_bevaluate: d_y[q] = sum_faces prod_{t fixed} b_{c_t}(x_t) f_face(x_S), each f_face through the
+ *   zero-boundary evaluation path.  All device calls are asynchronous on `stream`. */
+typedef struct sg_bgrid_s *sg_bgrid;
+sg_status sg_bcreate(int32_t d, int32_t n, sg_bgrid *out, uint64_t *num_points);
+sg_status sg_bdestroy(sg_bgrid g);
+sg_status sg_bface(sg_bgrid g, uint32_t face, uint32_t *free_mask, uint32_t *fixed_bits, uint64_t *first,
+                   uint64_t *count);
+sg_status sg_bcoords_device(sg_bgrid g, void *d_x, sg_dtype dt, void *stream);
+sg_status sg_bhierarchize(sg_bgrid g, void *d_values, sg_dtype dt, void *stream);
+sg_status sg_bevaluate(sg_bgrid g, const void *d_alpha, const void *d_x, uint64_t m, void *d_y, sg_dtype dt,
+                       void *stream);
+
 /* End-to-end evaluation from HOST buffers: copies h_x (m x d) to the device,
  * evaluates as sg_evaluate, copies the m results to h_y.  d_alpha is on the
  * device.  Device buffers are allocated stream-ordered.  The three steps run

@@ -11,5 +11,5 @@ from ._sg import (SG_EVAL_PRESORTED, SG_F32, SG_F64, SgError, sg_build_info, sg_
                   sg_gp2idx_device, sg_grid_coords_device, sg_hierarchize, sg_idx2gp, sg_idx2gp_device,
                   sg_kernel_launch_count, sg_profile_enable, sg_profile_read, sg_sfc_order, sg_evaluate_ordered, sg_evaluate_plane,
                   sg_plane_workspace_bytes, sg_part_bounds, sg_evaluate_part)
-from .grid import Grid  # noqa: F401
+from .grid import BoundaryGrid, Grid  # noqa: F401
 from .multi import evaluate_distributed, evaluate_sharded_grid, partition  # noqa: F401

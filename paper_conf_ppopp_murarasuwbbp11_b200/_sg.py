@@ -57,6 +57,12 @@ _SIGS = {
     "sg_evaluate_ordered": [_p, _p, _p, _u64, _p, _u64, _u64, _p, ctypes.c_int, _p],
     "sg_plane_workspace_bytes": [_p, _u32, _u32, ctypes.c_int, ctypes.POINTER(_sz)],
     "sg_part_bounds": [_p, _u32, _u32, ctypes.POINTER(_u64), ctypes.POINTER(_u64)],
+    "sg_bcreate": [_i32, _i32, ctypes.POINTER(_p), ctypes.POINTER(_u64)],
+    "sg_bdestroy": [_p],
+    "sg_bface": [_p, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32), ctypes.POINTER(_u64), ctypes.POINTER(_u64)],
+    "sg_bcoords_device": [_p, _p, ctypes.c_int, _p],
+    "sg_bhierarchize": [_p, _p, ctypes.c_int, _p],
+    "sg_bevaluate": [_p, _p, _p, _u64, _p, ctypes.c_int, _p],
     "sg_evaluate_part": [_p, _p, _u32, _u32, _p, _u64, _p, _p, ctypes.c_int, ctypes.c_int, _p],
     "sg_evaluate_plane": [_p, _p, _p, _p, _p, _u32, _u32, _p, ctypes.c_int, _u32, _p, _sz, _p],
 }
@@ -264,6 +270,37 @@ def sg_evaluate_part(g, alpha_part: torch.Tensor, parts: int, part: int, x: torc
     ap = _dev(alpha_part, "alpha_part") if alpha_part.numel() else None
     _check(lib.sg_evaluate_part(g, ap, parts, part, _dev(x, "x"), x.shape[0], pp, _dev(y, "y"), 1 if accumulate else 0,
                                 _dtype_code(x), _stream(stream)), "sg_evaluate_part")
+
+
+def sg_bcreate(d: int, n: int):
+    h = ctypes.c_void_p()
+    N = ctypes.c_uint64()
+    _check(lib.sg_bcreate(d, n, ctypes.byref(h), ctypes.byref(N)), "sg_bcreate")
+    return h, int(N.value)
+
+
+def sg_bdestroy(g) -> None:
+    _check(lib.sg_bdestroy(g), "sg_bdestroy")
+
+
+def sg_bface(g, face: int) -> tuple[int, int, int, int]:
+    m, b, f, c = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib.sg_bface(g, face, ctypes.byref(m), ctypes.byref(b), ctypes.byref(f), ctypes.byref(c)), "sg_bface")
+    return int(m.value), int(b.value), int(f.value), int(c.value)
+
+
+def sg_bcoords_device(g, x: torch.Tensor, stream=None) -> None:
+    _check(lib.sg_bcoords_device(g, _dev(x, "x"), _dtype_code(x), _stream(stream)), "sg_bcoords_device")
+
+
+def sg_bhierarchize(g, values: torch.Tensor, stream=None) -> None:
+    _check(lib.sg_bhierarchize(g, _dev(values, "values"), _dtype_code(values), _stream(stream)), "sg_bhierarchize")
+
+
+def sg_bevaluate(g, alpha: torch.Tensor, x: torch.Tensor, y: torch.Tensor, stream=None) -> None:
+    _check_batch(alpha, x, y)
+    _check(lib.sg_bevaluate(g, _dev(alpha, "alpha"), _dev(x, "x"), x.shape[0], _dev(y, "y"), _dtype_code(x),
+                            _stream(stream)), "sg_bevaluate")
 
 
 def sg_evaluate_host(g, alpha: torch.Tensor, x_host, y_host, flags: int = 0, stream=None) -> None:

@@ -132,3 +132,45 @@ class Grid:
             y_host = torch.empty(x_host.shape[0], dtype=x_host.dtype, pin_memory=True)
         _sg.sg_evaluate_host(self._h, alpha, x_host, y_host, _sg.SG_EVAL_PRESORTED if presorted else 0)
         return y_host
+
+
+class BoundaryGrid:
+    """Sparse grid with non-zero boundary (NEXT-2; paper Sec. 4.4, Fig. 7): the 3^d faces, each a
+    zero-boundary sparse grid of its free dimensions (include/sg.h "NON-ZERO boundary")."""
+
+    def __init__(self, d: int, n: int):
+        self._h, self.num_points = _sg.sg_bcreate(d, n)
+        self.d, self.n = d, n
+        self.num_faces = 3 ** d
+
+    def close(self):
+        if getattr(self, "_h", None) is not None:
+            _sg.sg_bdestroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def face(self, f: int) -> dict:
+        mask, bits, first, count = _sg.sg_bface(self._h, f)
+        return dict(free=[t for t in range(self.d) if mask >> t & 1], fixed_bits=bits, first=first, count=count)
+
+    def coords(self, dtype=torch.float64, device="cuda") -> torch.Tensor:
+        x = torch.empty((self.num_points, self.d), dtype=dtype, device=device)
+        _sg.sg_bcoords_device(self._h, x)
+        return x
+
+    def hierarchize_(self, values: torch.Tensor) -> torch.Tensor:
+        if values.numel() != self.num_points:
+            raise ValueError(f"values has {values.numel()} entries, the grid {self.num_points} points")
+        _sg.sg_bhierarchize(self._h, values)
+        return values
+
+    def evaluate(self, alpha: torch.Tensor, x: torch.Tensor, out: torch.Tensor | None = None) -> torch.Tensor:
+        _sg._check_batch(alpha, x, out, self.num_points, self.d)
+        y = out if out is not None else torch.empty(x.shape[0], dtype=x.dtype, device=x.device)
+        _sg.sg_bevaluate(self._h, alpha, x.contiguous(), y)
+        return y

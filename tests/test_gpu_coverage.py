@@ -317,3 +317,50 @@ def test_gloo_world2_sharded_grid_on_one_gpu(P, torch, tmp_path):
     y0, y1 = np.load(tmp_path / "y0.npy"), np.load(tmp_path / "y1.npy")
     assert np.array_equal(y0, y1)  # every rank holds the reduced result
     np.testing.assert_allclose(y0, ref, rtol=1e-12, atol=0)  # positive surpluses: plain relative error
+
+
+# ----------------------------------------------------------------- non-zero boundary (NEXT-2)
+@pytest.mark.parametrize("d,n,dt", [(1, 5, "f64"), (2, 4, "f64"), (3, 3, "f64"), (3, 5, "f64"), (4, 3, "f64"),
+                                    (2, 6, "f32")])
+def test_boundary_grid_vs_oracle(P, torch, oracle, d, n, dt):
+    """BoundaryGrid (sg_bcreate / sg_bcoords_device / sg_bhierarchize / sg_bevaluate) against the pinned
+    boundary oracle: layout and coordinates exact, surpluses bit-exact (fp64), evaluations within the
+    normwise tolerance at random points, grid points, boundary points and outside the cube."""
+    from oracle import boundary as OB
+    g = P.BoundaryGrid(d, n)
+    assert g.num_points == OB.num_points(d, n)
+    xp, _, _, _ = OB.points(d, n)
+    for f, (S_, c) in enumerate(OB.faces(d)):
+        fc = g.face(f)
+        assert fc["free"] == list(S_)
+        assert fc["fixed_bits"] == sum(b << k for k, b in enumerate(c))
+    T = tdt(torch, dt)
+    x = g.coords(dtype=T)
+    np.testing.assert_array_equal(x.cpu().numpy().astype(np.float64), xp)
+    f = np.sin(3.0 * xp.sum(1)) + 0.5 * xp[:, 0] * (1.0 - 0.3 * xp[:, -1]) + 0.25
+    vals = torch.from_numpy(f).to(T).cuda()
+    alpha = g.hierarchize_(vals.clone())
+    want = OB.hierarchize(d, n, vals.cpu().numpy().astype(np.float64))
+    if dt == "f64":
+        np.testing.assert_array_equal(alpha.cpu().numpy(), want)
+    else:
+        np.testing.assert_allclose(alpha.cpu().numpy(), want, rtol=0, atol=1e-5 * np.abs(want).max() * d * n)
+    q = np.concatenate([S.queries(d, 300, 17 + d), xp[:: max(1, len(xp) // 50)],
+                        np.full((1, d), 0.0), np.full((1, d), 1.0), np.full((1, d), 1.5)])
+    qt = torch.from_numpy(q).to(T).cuda()
+    y = g.evaluate(alpha, qt).cpu().numpy().astype(np.float64)
+    yo, ao = OB.evaluate(d, n, alpha.cpu().numpy().astype(np.float64), qt.cpu().numpy().astype(np.float64))
+    check_eval(y, yo, ao, TOL[dt], f"boundary d={d} n={n} {dt}")
+    assert y[-1] == 0.0  # outside the cube
+
+
+def test_boundary_grid_reproduces_multilinear(P, torch):
+    """The boundary basis spans the multilinear functions: f_s = f everywhere for f = prod (a_t + b_t x_t)."""
+    d, n = 3, 5
+    g = P.BoundaryGrid(d, n)
+    a = torch.tensor([1.0, 0.5, 2.0], dtype=torch.float64, device="cuda")
+    b = torch.tensor([0.3, -0.2, 1.1], dtype=torch.float64, device="cuda")
+    ml = lambda z: torch.prod(a + b * z, dim=1)
+    alpha = g.hierarchize_(ml(g.coords()))
+    q = S.queries_torch(d, 5000, 9, device="cuda")
+    torch.testing.assert_close(g.evaluate(alpha, q), ml(q), rtol=1e-13, atol=1e-14)
