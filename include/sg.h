@@ -241,6 +241,10 @@ sg_status sg_evaluate_host(sg_grid g, const void *d_alpha, const void *h_x, uint
  * for the bench's gpu_launches count). */
 uint64_t sg_kernel_launch_count(void);
 
+/* Test instrumentation: the (mangled) names of the distinct kernels the library launched since load,
+ * newline-separated, into buf (at most len bytes incl. the terminating 0); returns the bytes needed. */
+size_t sg_launched_kernels(char *buf, size_t len);
+
 /* Kernel timing instrumentation.  While enabled (on != 0), every evaluation
  * kernel launch and every hierarchization pass is bracketed by CUDA events
  * recorded on the launching stream.  sg_profile_read synchronizes on those

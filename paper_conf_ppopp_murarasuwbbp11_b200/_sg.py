@@ -77,6 +77,8 @@ lib.sg_profile_read.argtypes = [ctypes.POINTER(ctypes.c_double), ctypes.POINTER(
 lib.sg_profile_read.restype = ctypes.c_int
 lib.sg_kernel_launch_count.restype = _u64
 lib.sg_kernel_launch_count.argtypes = []
+lib.sg_launched_kernels.restype = _sz
+lib.sg_launched_kernels.argtypes = [ctypes.c_char_p, _sz]
 for _name in ("sg_last_error", "sg_build_info"):
     getattr(lib, _name).restype = ctypes.c_char_p
     getattr(lib, _name).argtypes = []
@@ -85,7 +87,7 @@ lib.sg_status_string.argtypes = [ctypes.c_int]
 
 #: every entry point declared in include/sg.h
 EXPORTS = tuple(_SIGS) + ("sg_kernel_launch_count", "sg_status_string", "sg_last_error", "sg_build_info",
-                          "sg_profile_enable", "sg_profile_read")
+                          "sg_profile_enable", "sg_profile_read", "sg_launched_kernels")
 
 
 class SgError(RuntimeError):
@@ -315,6 +317,14 @@ def sg_evaluate_host(g, alpha: torch.Tensor, x_host, y_host, flags: int = 0, str
 
 def sg_kernel_launch_count() -> int:
     return int(lib.sg_kernel_launch_count())
+
+
+def sg_launched_kernels() -> list[str]:
+    """Mangled names of the distinct libsg kernels launched since load (test instrumentation)."""
+    need = int(lib.sg_launched_kernels(None, 0))
+    buf = ctypes.create_string_buffer(need)
+    lib.sg_launched_kernels(buf, need)
+    return [s for s in buf.value.decode().split("\n") if s]
 
 
 def sg_build_info() -> str:

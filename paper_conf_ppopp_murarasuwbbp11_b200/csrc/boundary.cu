@@ -368,7 +368,7 @@ sg_status sg_bcoords_device(sg_bgrid g, void* d_x, sg_dtype dt, void* stream) {
     else
       k_embed<float><<<grid_for(f.count), kThreads, 0, s>>>((const float*)tmp, f.count, d, f.mask, f.bits,
                                                             (float*)d_x + f.first * d);
-    st = launched("k_embed");
+    st = launched("k_embed", dt == SG_F64 ? (const void*)k_embed<double> : (const void*)k_embed<float>);
     if (st != SG_OK) break;
   }
   cudaFreeAsync(tmp, s);
@@ -417,7 +417,7 @@ sg_status sg_bhierarchize(sg_bgrid g, void* d_values, sg_dtype dt, void* stream)
         k_hier_family_b<float><<<(unsigned)tab.F, kThreads, smem, s>>>(
             n, tab.info, tab.first, tab.bases, tab.bbase, (float*)(v + f.first * es),
             (const float*)(v + g->faces[f0].first * es), (const float*)(v + g->faces[f1].first * es));
-      st = launched("k_hier_family_b");
+      st = launched("k_hier_family_b", dt == SG_F64 ? (const void*)k_hier_family_b<double> : (const void*)k_hier_family_b<float>);
       if (st != SG_OK) return st;
     }
   }
@@ -452,7 +452,7 @@ sg_status sg_bevaluate(sg_bgrid g, const void* d_alpha, const void* d_x, uint64_
     if (f.j > 0) {
       if (dt == SG_F64) k_project<double><<<grid_for(m), kThreads, 0, s>>>((const double*)d_x, m, d, f.mask, (double*)xs);
       else k_project<float><<<grid_for(m), kThreads, 0, s>>>((const float*)d_x, m, d, f.mask, (float*)xs);
-      st = launched("k_project");
+      st = launched("k_project", dt == SG_F64 ? (const void*)k_project<double> : (const void*)k_project<float>);
       if (st == SG_OK) st = sg_evaluate(g->sub[f.j], a + f.first * es, xs, m, yf, dt, 0, nullptr, 0, stream);
       if (st != SG_OK) break;
     } else {
@@ -464,7 +464,7 @@ sg_status sg_bevaluate(sg_bgrid g, const void* d_alpha, const void* d_x, uint64_
     else
       k_face_axpy<float><<<grid_for(m), kThreads, 0, s>>>((const float*)d_x, m, d, f.mask, f.bits, (const float*)yf,
                                                           (const float*)corner, (float*)d_y);
-    st = launched("k_face_axpy");
+    st = launched("k_face_axpy", dt == SG_F64 ? (const void*)k_face_axpy<double> : (const void*)k_face_axpy<float>);
     if (st != SG_OK) break;
   }
   cudaFreeAsync(xs, s);

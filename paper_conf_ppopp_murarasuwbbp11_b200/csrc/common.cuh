@@ -36,6 +36,13 @@ inline sg_status launched(const char* what) {
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? SG_OK : cuda_fail(e, what);
 }
+// the same, recording WHICH kernel was launched (sg_launched_kernels: test instrumentation that checks every
+// kernel in the library is exercised by the parity tests)
+void record_kernel(const void* func);
+inline sg_status launched(const char* what, const void* func) {
+  record_kernel(func);
+  return launched(what);
+}
 
 constexpr int kNumSMs = 148;
 

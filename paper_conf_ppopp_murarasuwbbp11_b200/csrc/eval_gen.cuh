@@ -254,7 +254,7 @@ sg_status launch_gen(const T* alpha, const T* x, const uint32_t* perm, uint64_t 
   if (st != SG_OK) return st;
   const unsigned blocks = (unsigned)((m + NT - 1) / NT);
   kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, n, y, j0, v0, j1, v1, b0, accumulate);
-  return launched("k_eval_gen");
+  return launched("k_eval_gen", (const void*)kern);
 }
 
 }  // namespace gen

@@ -85,7 +85,7 @@ sg_status launch_eval_simple(const sg_grid_s* g, const void* alpha, const void* 
   else
     k_eval_simple<float><<<(unsigned)blocks, kThreads, 0, s>>>(g->d_L, (const float*)alpha, (const float*)x, perm, m,
                                                                (float*)y);
-  return launched("k_eval_simple");
+  return launched("k_eval_simple", dt == SG_F64 ? (const void*)k_eval_simple<double> : (const void*)k_eval_simple<float>);
 }
 
 }  // namespace sg

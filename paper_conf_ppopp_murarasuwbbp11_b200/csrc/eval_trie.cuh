@@ -553,7 +553,7 @@ sg_status launch_range(const Layout& L, const T* alpha, const T* x, const uint32
   // the first launch of a call (group 0, all budgets) writes y, every later one accumulates
   const int accumulate = (J0 > 0 || KN::RMIN > 0) ? 1 : 0;
   kern<<<blocks, NT, smem, s>>>(alpha, x, perm, (uint32_t)m, L.n, (uint32_t)L.off[J0], accumulate, y);
-  return launched("k_eval_trie");
+  return launched("k_eval_trie", (const void*)kern);
 }
 
 }  // namespace trie

@@ -201,7 +201,7 @@ sg_status hier_table(const sg_grid_s* g, HierTab* tab) {
       for (int t = 0; t < d && st == SG_OK; ++t) {
         const unsigned blocks = (unsigned)((tab->F + kThreads - 1) / kThreads);
         k_hier_table<<<blocks, kThreads, 0, bs>>>(g->d_L, t, tab->F, in + (size_t)t * tab->F * 2, b + (size_t)t * nb);
-        st = launched("k_hier_table");
+        st = launched("k_hier_table", (const void*)k_hier_table<0>);
       }
       e = cudaStreamSynchronize(bs);
       cudaStreamDestroy(bs);
@@ -279,7 +279,7 @@ sg_status hierarchize_t(const sg_grid_s* g, T* v, cudaStream_t s) {
     for (int t = 0; t < d; ++t) {
       k_hier_family2<T><<<(unsigned)tab.F, kThreads, fam_bytes, s>>>(n, tab.info + (size_t)t * tab.F * 2,
                                                                        tab.base + (size_t)t * tab.nbase, v);
-      st = launched("k_hier_family2");
+      st = launched("k_hier_family2", (const void*)k_hier_family2<T>);
       if (st != SG_OK) return st;
     }
     return SG_OK;
@@ -294,7 +294,7 @@ sg_status hierarchize_t(const sg_grid_s* g, T* v, cudaStream_t s) {
   T* b = tmp;
   for (int t = 0; t < d; ++t) {
     k_hier_global<T><<<(unsigned)blocks, kThreads, 0, s>>>(g->d_L, t, a, b);
-    sg_status st = launched("k_hier_global");
+    sg_status st = launched("k_hier_global", (const void*)k_hier_global<T>);
     if (st != SG_OK) return st;
     T* c = a;
     a = b;

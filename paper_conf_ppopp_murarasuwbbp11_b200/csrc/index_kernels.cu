@@ -83,14 +83,14 @@ sg_status launch_gp2idx(const sg_grid_s* g, const int32_t* l, const int32_t* i, 
                         cudaStream_t s) {
   if (count == 0) return SG_OK;
   k_gp2idx<<<grid_for(count), kThreads, 0, s>>>(g->d_L, l, i, count, idx);
-  return launched("k_gp2idx");
+  return launched("k_gp2idx", (const void*)k_gp2idx);
 }
 
 sg_status launch_idx2gp(const sg_grid_s* g, const uint64_t* idx, uint64_t count, int32_t* l, int32_t* i,
                         cudaStream_t s) {
   if (count == 0) return SG_OK;
   k_idx2gp<<<grid_for(count), kThreads, 0, s>>>(g->d_L, idx, count, l, i);
-  return launched("k_idx2gp");
+  return launched("k_idx2gp", (const void*)k_idx2gp);
 }
 
 sg_status launch_coords(const sg_grid_s* g, uint64_t first, uint64_t count, void* x, sg_dtype dt, cudaStream_t s) {
@@ -99,7 +99,7 @@ sg_status launch_coords(const sg_grid_s* g, uint64_t first, uint64_t count, void
     k_coords<double><<<grid_for(count), kThreads, 0, s>>>(g->d_L, first, count, (double*)x);
   else
     k_coords<float><<<grid_for(count), kThreads, 0, s>>>(g->d_L, first, count, (float*)x);
-  return launched("k_coords");
+  return launched("k_coords", dt == SG_F64 ? (const void*)k_coords<double> : (const void*)k_coords<float>);
 }
 
 }  // namespace sg

@@ -107,7 +107,7 @@ sg_status launch_plane(const sg_grid_s* g, const void* alpha, const double* orig
   else
     k_plane_coords<float><<<(unsigned)blocks, kThreads, 0, s>>>(pa, d, width, height, ord, tiles_x, kx, ky,
                                                                  (float*)x, perm);
-  sg_status st = launched("k_plane_coords");
+  sg_status st = launched("k_plane_coords", dt == SG_F64 ? (const void*)k_plane_coords<double> : (const void*)k_plane_coords<float>);
   if (st != SG_OK) return st;
   return launch_evaluate(g, alpha, x, perm, m, img, dt, 0, s);
 }

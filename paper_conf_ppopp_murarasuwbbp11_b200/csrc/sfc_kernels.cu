@@ -125,7 +125,7 @@ sg_status launch_sfc_order(const sg_grid_s* g, const void* x, uint64_t m, sg_dty
     k_morton<double><<<(unsigned)blocks, kThreads, 0, s>>>((const double*)x, m, d, bits, cap, start, k0, v0);
   else
     k_morton<float><<<(unsigned)blocks, kThreads, 0, s>>>((const float*)x, m, d, bits, cap, start, k0, v0);
-  sg_status st = launched("k_morton");
+  sg_status st = launched("k_morton", dt == SG_F64 ? (const void*)k_morton<double> : (const void*)k_morton<float>);
   if (st != SG_OK) return st;
   // the sort is deterministic (stable LSD radix sort of (key, index) pairs): every rank that orders the same
   // batch gets the same permutation (ranks agree on one global order without communicating)

@@ -6,6 +6,8 @@
 #include <string.h>
 
 #include <mutex>
+#include <set>
+#include <string>
 #include <new>
 #include <vector>
 
@@ -16,6 +18,14 @@ namespace sg {
 std::atomic<uint64_t> g_launches{0};
 
 static thread_local char t_err[512] = "";
+
+// kernels launched since load (test instrumentation: sg_launched_kernels)
+static std::mutex g_kern_mu;
+static std::set<const void*> g_kernels;
+void record_kernel(const void* func) {
+  std::lock_guard<std::mutex> lk(g_kern_mu);
+  g_kernels.insert(func);
+}
 
 void set_error(const char* fmt, ...) {
   va_list ap;
@@ -590,6 +600,26 @@ sg_status sg_evaluate_host(sg_grid g, const void* d_alpha, const void* h_x, uint
 }
 
 uint64_t sg_kernel_launch_count(void) { return g_launches.load(); }
+
+size_t sg_launched_kernels(char* buf, size_t len) {
+  std::string names;
+  {
+    std::lock_guard<std::mutex> lk(g_kern_mu);
+    for (const void* f : g_kernels) {
+      const char* nm = nullptr;
+      if (cudaFuncGetName(&nm, f) == cudaSuccess && nm) {
+        names += nm;
+        names += '\n';
+      }
+    }
+  }
+  if (buf && len) {
+    const size_t k = names.size() < len - 1 ? names.size() : len - 1;
+    memcpy(buf, names.data(), k);
+    buf[k] = 0;
+  }
+  return names.size() + 1;
+}
 
 sg_status sg_profile_enable(int on) {
   g_prof_on.store(on ? 1 : 0);

@@ -51,4 +51,18 @@ if __name__ == "__main__":
     run(7, 5, torch.float32, generic=True)
     run(3, 14, m=64)
     run(1, 17, m=64)
+    # visualization slice, sharded-grid parts, boundary grid
+    g = P.Grid(3, 8)
+    a = g.hierarchize_(S.f_A_torch(g.coords()))
+    g.render_plane(a, [0.0, 0.0, 0.3], [1 / 64, 0.0, 0.0], [0.0, 1 / 32, 0.0], 64, 32, order=1)
+    x = S.queries_torch(3, 500, 3, device="cuda")
+    y = torch.zeros(500, dtype=torch.float64, device="cuda")
+    for r in range(3):
+        first, count = g.part_bounds(3, r)
+        g.evaluate_part(a[first:first + count].clone(), 3, r, x, out=y, accumulate=True)
+    bg = P.BoundaryGrid(3, 4)
+    ba = bg.hierarchize_(S.f_A_torch(bg.coords()) + 1.0)
+    bg.evaluate(ba, x)
+    torch.cuda.synchronize()
+    print("plane / parts / boundary: ok", flush=True)
     print("sanitize run complete")

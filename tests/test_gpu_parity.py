@@ -135,12 +135,18 @@ def test_hierarchize_table_reuse_and_fp32(P, torch, oracle):
     np.testing.assert_allclose(got32, want, rtol=0, atol=64 * d * np.finfo(np.float32).eps * np.abs(v32).max())
 
 
-@pytest.mark.parametrize("d,n", [(1, 17), (2, 15)])
-def test_hierarchize_large_families_fallback(P, torch, oracle, d, n):
+@pytest.mark.parametrize("d,n,dt", [(1, 17, "f64"), (2, 15, "f64"), (1, 17, "f32")])
+def test_hierarchize_large_families_fallback(P, torch, oracle, d, n, dt):
     # 2^n - 1 values per pole family exceed shared memory: global ping-pong kernel
     g = P.Grid(d, n)
     xs = oracle.coords(d, n)
     v = S.f_A(xs) + 0.25 * np.cos(5.0 * xs.sum(1))
+    if dt == "f32":
+        v32 = v.astype(np.float32)
+        want = oracle.hierarchize(d, n, v32.astype(np.float64))
+        got = g.hierarchize_(torch.from_numpy(v32).cuda()).cpu().numpy().astype(np.float64)
+        np.testing.assert_allclose(got, want, rtol=0, atol=64 * d * np.finfo(np.float32).eps * np.abs(v32).max())
+        return
     want = oracle.hierarchize(d, n, v)
     got = g.hierarchize_(torch.from_numpy(v).cuda()).cpu().numpy()
     np.testing.assert_array_equal(got, want)
