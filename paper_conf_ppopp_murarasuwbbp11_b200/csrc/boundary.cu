@@ -350,6 +350,7 @@ sg_status sg_bcoords_device(sg_bgrid g, void* d_x, sg_dtype dt, void* stream) {
     return SG_ERR_NODEV;
   }
   if (dt != SG_F64 && dt != SG_F32) return SG_ERR_DTYPE;
+  NvtxRange nvtx("sg_bcoords_device");
   cudaStream_t s = (cudaStream_t)stream;
   const size_t es = dt_size(dt);
   const int d = g->d;
@@ -382,6 +383,7 @@ sg_status sg_bhierarchize(sg_bgrid g, void* d_values, sg_dtype dt, void* stream)
     return SG_ERR_NODEV;
   }
   if (dt != SG_F64 && dt != SG_F32) return SG_ERR_DTYPE;
+  NvtxRange nvtx("sg_bhierarchize");
   cudaStream_t s = (cudaStream_t)stream;
   const size_t es = dt_size(dt);
   const int n = g->n;
@@ -433,6 +435,7 @@ sg_status sg_bevaluate(sg_bgrid g, const void* d_alpha, const void* d_x, uint64_
   }
   if (dt != SG_F64 && dt != SG_F32) return SG_ERR_DTYPE;
   if (m == 0) return SG_OK;
+  NvtxRange nvtx("sg_bevaluate");
   cudaStream_t s = (cudaStream_t)stream;
   const size_t es = dt_size(dt);
   const int d = g->d;

@@ -3,6 +3,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include <atomic>
 #include <mutex>
 
@@ -45,6 +47,15 @@ inline sg_status launched(const char* what, const void* func) {
 }
 
 constexpr int kNumSMs = 148;
+
+// NVTX range around one ABI call (header-only NVTX3: a no-op unless a profiler is attached), so that
+// nsys/ncu timelines show the path's steps (a1 ordering, a2-a6 evaluation, a7 hierarchization, NEXT rows)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 // Function attributes are per device: opt a kernel into `smem` bytes of dynamic
 // shared memory (and an L1/shared carveout, percent; < 0 = leave it) once per

@@ -363,6 +363,7 @@ sg_status sg_hierarchize(sg_grid g, void* d_values, sg_dtype dt, void* stream) {
   if (!dtype_ok(dt)) return SG_ERR_DTYPE;
   if (!d_values) return SG_ERR_ARG;
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_hierarchize");
   return launch_hierarchize(g, d_values, dt, (cudaStream_t)stream);
 }
 
@@ -389,6 +390,7 @@ sg_status sg_evaluate(sg_grid g, const void* d_alpha, const void* d_x, uint64_t 
     return SG_ERR_ARG;
   }
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_evaluate");
   cudaStream_t s = (cudaStream_t)stream;
   const uint32_t* perm = nullptr;
   void* own_ws = nullptr;
@@ -423,6 +425,7 @@ sg_status sg_sfc_order(sg_grid g, const void* d_x, uint64_t m, sg_dtype dt, uint
     return SG_ERR_ARG;
   }
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_sfc_order");
   cudaStream_t s = (cudaStream_t)stream;
   void* own_ws = nullptr;
   if (!d_workspace) {
@@ -456,6 +459,7 @@ sg_status sg_evaluate_ordered(sg_grid g, const void* d_alpha, const void* d_x, u
     return SG_ERR_ARG;
   }
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_evaluate_ordered");
   const size_t es = dtype_size(dt);
   if (d_perm)  // positions first..first+count-1 of the order; x and y indexed by the query's input position
     return launch_evaluate(g, d_alpha, d_x, d_perm + first, count, d_y, dt, SG_EVAL_PRESORTED, (cudaStream_t)stream);
@@ -489,6 +493,7 @@ sg_status sg_evaluate_plane(sg_grid g, const void* d_alpha, const double* origin
     return SG_ERR_ARG;
   }
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_evaluate_plane");
   cudaStream_t s = (cudaStream_t)stream;
   const size_t need = plane_workspace_bytes(g->L.d, m, dtype_size(dt));
   void* own = nullptr;
@@ -539,6 +544,7 @@ sg_status sg_evaluate_part(sg_grid g, const void* d_alpha_part, uint32_t parts, 
   PartRange pr;
   part_range(g->L, parts, part, &pr);
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_evaluate_part");
   cudaStream_t s = (cudaStream_t)stream;
   if (pr.count == 0) {  // an empty part adds nothing; without accumulate y is defined as 0
     if (!accumulate) {
@@ -574,6 +580,7 @@ sg_status sg_evaluate_host(sg_grid g, const void* d_alpha, const void* h_x, uint
   if (m == 0) return SG_OK;
   if (!d_alpha || !h_x || !h_y) return SG_ERR_ARG;
   DeviceGuard guard(g->device);
+  NvtxRange nvtx("sg_evaluate_host");
   cudaStream_t s = (cudaStream_t)stream;
   const size_t xb = m * (size_t)g->L.d * dtype_size(dt), yb = m * dtype_size(dt);
   void *dx = nullptr, *dy = nullptr;
