@@ -78,6 +78,15 @@ struct Knobs {
   // RMIN prunes trie nodes (sub-tries of level sum < RMIN) but does not filter blocks: the complement of
   // a launch with a larger INNER and RMAX = RMIN - 1 (whose blocks are exactly those sub-tries)
   static constexpr bool RMIN_NODES_ONLY = false;
+  // experiment builds only: shared-memory hat rows of the block dimensions 2..INNER-1 for all NM levels
+  // (r02 v8) instead of the RMAX + 1 levels a block can read (a launch of small blocks then takes
+  // 18 KB less shared memory per CTA, and the SM keeps that much more L1 for the surplus gathers)
+  static constexpr bool TAB_ALL = false;
+  // level-0 hat values of the block dimensions 2..INNER-1 in registers (read in every block)
+  static constexpr bool H0 = false;
+  // hat values of dimension I (the innermost trie dimension) by doubling along its level loop, like the
+  // dimensions above it, instead of a shared-memory row per level (NM - 1 fewer rows: more L1)
+  static constexpr bool IDBL = false;
 };
 struct KnobsS0 : Knobs {
   static constexpr bool S0 = true;
@@ -92,10 +101,14 @@ struct Trie {
   static constexpr bool CST = KN::CST;
   // shared memory, [row][lane]: hat values of dimensions 2, 3 (read per block / slab), of
   // dimension I (per dimension-I node), then x of dimensions I+1..D-1
-  static constexpr int SM_IN = (I > 2 ? I - 2 : 0) * NM;  // hat rows of dimensions 2 .. I-1
-  static constexpr int SM_PH = O > 0 ? NM : 0;
-  static constexpr int SM_X = O > 1 ? O - 1 : 0;
-  static constexpr int xrow(int t) { return t - I - 1; }
+  // levels of the block dimensions' hat rows: a block of budget R <= RMAX reads levels 0..R
+  static constexpr int PHB = (KN::TAB_ALL || KN::RMAX + 1 >= NM) ? NM : KN::RMAX + 1;
+  static constexpr int SM_IN = (I > 2 ? I - 2 : 0) * PHB;  // hat rows of dimensions 2 .. I-1
+  static constexpr bool H0 = KN::H0 && I > 2;
+  static constexpr bool IDBL = KN::IDBL && O > 0;
+  static constexpr int SM_PH = (O > 0 && !IDBL) ? NM : 0;
+  static constexpr int SM_X = IDBL ? O : (O > 1 ? O - 1 : 0);
+  static constexpr int xrow(int t) { return IDBL ? t - I : t - I - 1; }
   // S0: suffix products P0[t] = prod_{u <= t} phi_0(x_u), t = I..D-1, so that a
   // sub-trie whose level budget is exhausted (every level of dimensions t..0
   // is 0: one term, one surplus) costs one gather and one FMA instead of a
@@ -121,6 +134,7 @@ struct Trie {
     T d01[D01 ? PHN * (PHN + 1) / 2 : 1];  // D01: phi_0(r - l1) phi_1(l1) at index r (r + 1) / 2 + l1
     uint32_t ct[CST ? NM : 1];             // CST: C_J[u] = (k_0 digits of level J above bit u) | (K_1 >> (NM-1-u))
     T ph23[H23 ? 2 : 1][H23 ? PHN : 1];  // H23: hat values of dimensions 2, 3 (registers)
+    T h0[H0 ? 3 : 1];                      // H0: level-0 hat values of dimensions 2, 3, 4 (registers)
     uint32_t K[D];
     double res;  // the query's sum over the blocks: fp64 also for fp32 storage (reading G13: a long
                  // sequential fp32 accumulation would lose ~sqrt(#blocks) ulps of fp32)
@@ -196,8 +210,9 @@ struct Trie {
         ph2[l] = c.ph23[0][H23 ? l : 0];
         if constexpr (!LZ3) ph3[l] = c.ph23[H23 ? 1 : 0][H23 ? l : 0];
       } else {
-        ph2[l] = (NI >= 3) ? phs_at(c.phs, 0 * NM + l) : T(1);
-        if constexpr (!LZ3) ph3[l] = (NI >= 4) ? phs_at(c.phs, 1 * NM + l) : T(1);
+        ph2[l] = (NI >= 3) ? ((H0 && l == 0) ? c.h0[0] : phs_at(c.phs, 0 * PHB + l)) : T(1);
+        if constexpr (!LZ3)
+          ph3[l] = (NI >= 4) ? ((H0 && l == 0) ? c.h0[H0 ? 1 : 0] : phs_at(c.phs, 1 * PHB + l)) : T(1);
       }
     }
     // INNER = 5: hat values of dimension 4 for levels 0..R, from shared memory
@@ -205,7 +220,7 @@ struct Trie {
     uint32_t k4 = 0;
     if constexpr (NI >= 5) {
 #pragma unroll
-      for (int l = 0; l <= R; ++l) ph4[l] = phs_at(c.phs, 2 * NM + l);
+      for (int l = 0; l <= R; ++l) ph4[l] = (H0 && l == 0) ? c.h0[H0 ? 2 : 0] : phs_at(c.phs, 2 * PHB + l);
       asm volatile("mov.b32 %0, %1;" : "=r"(k4) : "r"(c.K[NI > 4 ? 4 : 0]));
     }
     T acc = T(0);
@@ -254,7 +269,7 @@ struct Trie {
           acc3 = (NI >= 3) ? fma(acc2, ph2[l2], acc3) : acc2;
         }
         if constexpr (NI >= 4) {
-          const T h3 = LZ3 ? phs_at(c.phs, 1 * NM + l3) : ph3[LZ3 ? 0 : l3];
+          const T h3 = LZ3 ? phs_at(c.phs, 1 * PHB + l3) : ph3[LZ3 ? 0 : l3];
           acc4 = fma(acc3, h3, acc4);
         } else {
           acc4 = acc3;
@@ -295,13 +310,13 @@ struct Trie {
 
   // dimension I at compile-time budget B: levels l = L .. B unrolled into one basic block
   template <int J, int B, int L>
-  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod) {
+  static __device__ __forceinline__ void inner_unrolled(Ctx& c, uint32_t P, T prod, T u) {
     if constexpr (L <= B) {
       constexpr int SG = J - B;
-      const T ph = phs_at(c.phs, SM_IN + L);
+      const T ph = IDBL ? hat_u(u) : phs_at(c.phs, SM_IN + L);
       const uint32_t kt = c.K[I] >> (NM - 1 - L);
       block<J, B - L>(c, P | (kt << SG), prod * ph);
-      inner_unrolled<J, B, L + 1>(c, P, prod);
+      inner_unrolled<J, B, L + 1>(c, P, prod, IDBL ? dbl_u(u) : u);
     }
   }
 
@@ -317,7 +332,7 @@ struct Trie {
     } else if constexpr (t < I) {
       block<J, B>(c, P, prod);
     } else if constexpr (t == I) {
-      inner_unrolled<J, B, 0>(c, P, prod);
+      inner_unrolled<J, B, 0>(c, P, prod, IDBL ? c.xs[0] : T(0));
     } else {
       static_assert(B == 0, "only budget-0 sub-tries above dimension I are straight-line");
       // level 0 of dimension t: digit of length 0, hat phi_0(x_t)
@@ -343,13 +358,13 @@ struct Trie {
   // tail of dimension I at run-time budget B: the blocks R = RT .. 0
   // (l_I = B - R), merged into one basic block
   template <int J, int RT>
-  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod) {
+  static __device__ __forceinline__ void inner_tail(Ctx& c, int B, uint32_t P, T prod, T u) {
     if constexpr (RT >= 0) {
       const int lt = B - RT;
-      const T ph = phs_at(c.phs, SM_IN + lt);
+      const T ph = IDBL ? hat_u(u) : phs_at(c.phs, SM_IN + lt);
       const uint32_t kt = c.K[I] >> (NM - 1 - lt);
       block<J, RT>(c, P | (kt << (J - B)), prod * ph);
-      inner_tail<J, RT - 1>(c, B, P, prod);
+      inner_tail<J, RT - 1>(c, B, P, prod, IDBL ? dbl_u(u) : u);
     }
   }
 
@@ -412,12 +427,14 @@ struct Trie {
         inner_dispatch<J>(c, B, P, prod);
         return;
       }
+      T u = IDBL ? c.xs[0] : T(0);  // IDBL: u = 2^lt x_I - k_I(lt) along the level loop
       for (int lt = 0; lt < B - kTail; ++lt) {
-        const T ph = phs_at(c.phs, SM_IN + lt);
+        const T ph = IDBL ? hat_u(u) : phs_at(c.phs, SM_IN + lt);
         const uint32_t kt = c.K[I] >> (NM - 1 - lt);
         leaf<J>(c, B - lt, P | (kt << SG), prod * ph);
+        if constexpr (IDBL) u = dbl_u(u);
       }
-      inner_tail<J, kTail>(c, B, P, prod);
+      inner_tail<J, kTail>(c, B, P, prod, u);
     } else {
       if (B == 0) {
         flat<J, t, 0>(c, P, prod);
@@ -499,7 +516,7 @@ __global__ void __launch_bounds__(NT, MINB)
       const long long bits = __double_as_longlong(r) | ((long long)(c1 & 1u) << 63);
       sm[(TR::SM_IN + TR::SM_PH + TR::SM_X + TR::SM_S0 + t) * NT + tid] = (T)__longlong_as_double(bits);
     }
-    if (t <= I) {
+    if (t < I || (t == I && !TR::IDBL)) {
 #pragma unroll
       for (int l = 0; l < NM; ++l) {
         uint32_t cell;
@@ -512,7 +529,10 @@ __global__ void __launch_bounds__(NT, MINB)
         } else if (TR::H23 && t < 4 && l < TR::PHN) {
           c.ph23[TR::H23 ? t - 2 : 0][TR::H23 && l < TR::PHN ? l : 0] = h;
         }
-        else if (t < I) sm[((t - 2) * NM + l) * NT + tid] = h;
+        else if (t < I) {
+          if (l < TR::PHB) sm[((t - 2) * TR::PHB + (l < TR::PHB ? l : 0)) * NT + tid] = h;
+          if (TR::H0 && l == 0) c.h0[TR::H0 ? (t < 5 ? t - 2 : 0) : 0] = h;
+        }
         else sm[(TR::SM_IN + l) * NT + tid] = h;
       }
     } else {

@@ -6,7 +6,11 @@
 // warps/SM (128 registers); the large-block launch (blocks over dimensions 0..3, 12 warps/SM) prunes
 // exactly those sub-tries.  Groups 0-6 run as small blocks (R <= 6) at 16 warps/SM.  Measured +8% (split
 // at 4 dimensions) and +3% more (5 inner dimensions for the small blocks) over one launch per group at 12
-// warps/SM (profiles/r02_split.txt).  Split across files only so that nvcc compiles them in parallel.
+// warps/SM (profiles/r02_split.txt).  v9: the small-block launches run as 256-thread CTAs (2 per SM:
+// 8 warps of neighbouring queries share the SM's L1) with hat rows of dimensions 2..4 only up to level
+// RMAX (18 KB less shared memory per 128 queries, so more L1) and the level-0 hats of dimensions 2..4 in
+// registers: +4.2%, +2.5% and +1.2% (profiles/r02_v9.txt).  Split across files only so that nvcc
+// compiles them in parallel.
 #include "eval_trie.cuh"
 
 namespace sg {
@@ -17,6 +21,7 @@ template <int RL>
 struct KLow : trie::Knobs {
   static constexpr int RMAX = RL;
   static constexpr int INNER = 5;
+  static constexpr bool H0 = true;  // level-0 hats of dimensions 2..4 in registers (+1.2%, profiles/r02_v9.txt)
 };
 // large blocks: blocks over dimensions 0..3 of every dimension-4 node with budget > RL (exactly the
 // complement: the nodes of budget <= RL are the small-block launch's blocks)
@@ -31,10 +36,10 @@ sg_status trie_d10n11_a(const Layout& L, const double* a, const double* x, const
                         cudaStream_t s) {
   using namespace d10;
   sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 0, 6, KLow<6>>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 7, 7, KLow<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 256, 2, 0, 6, KLow<6>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 256, 2, 7, 7, KLow<4>>(L, a, x, p, m, y, s);
   if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 7, 7, KHigh<4>>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 8, 8, KLow<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 256, 2, 8, 8, KLow<4>>(L, a, x, p, m, y, s);
   if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 8, 8, KHigh<4>>(L, a, x, p, m, y, s);
   return st;
 }

@@ -11,6 +11,7 @@ template <int RL>
 struct KLow : trie::Knobs {
   static constexpr int RMAX = RL;
   static constexpr int INNER = 5;
+  static constexpr bool H0 = true;  // level-0 hats of dimensions 2..4 in registers (+1.2%, profiles/r02_v9.txt)
 };
 // large blocks: blocks over dimensions 0..3 of every dimension-4 node with budget > RL (exactly the
 // complement: the nodes of budget <= RL are the small-block launch's blocks)
@@ -25,9 +26,9 @@ sg_status trie_d10n11_b(const Layout& L, const double* a, const double* x, const
                         cudaStream_t s) {
   using namespace d10b;
   sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 9, 9, KLow<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 256, 2, 9, 9, KLow<4>>(L, a, x, p, m, y, s);
   if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 9, 9, KHigh<4>>(L, a, x, p, m, y, s);
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 4, 10, 10, KLow<4>>(L, a, x, p, m, y, s);
+  if (st == SG_OK) st = trie::launch_range<double, 10, 11, 256, 2, 10, 10, KLow<4>>(L, a, x, p, m, y, s);
   if (st == SG_OK) st = trie::launch_range<double, 10, 11, 128, 3, 10, 10, KHigh<4>>(L, a, x, p, m, y, s);
   return st;
 }

@@ -1,0 +1,3 @@
+// GOT: r02 v9 experiment variant (exp_v9.cuh)
+#include "exp_v9.cuh"
+SG_V9(exp_GOT, false, false, true, 256, 2, 128, 3)

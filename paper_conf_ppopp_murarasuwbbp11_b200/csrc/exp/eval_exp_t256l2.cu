@@ -1,0 +1,3 @@
+// T256L2: r02 v9 experiment variant (exp_v9.cuh)
+#include "exp_v9.cuh"
+SG_V9(exp_T256L2, false, false, false, 256, 2, 192, 2)
