@@ -297,18 +297,44 @@ def run_sg(args, rank, world, local_rank):
 
         step_e2e()
         barrier()
-        ev0.record(stream)
         e2e_steps = max(1, min(args.steps, args.e2e_steps))
-        for _ in range(e2e_steps):
+        evk = [torch.cuda.Event(enable_timing=True) for _ in range(e2e_steps + 1)]
+        ev0.record(stream)
+        evk[0].record(stream)
+        for k in range(e2e_steps):
             step_e2e()
+            evk[k + 1].record(stream)
         ev1.record(stream)
         barrier()
         e2e_ms = max_over_ranks(ev0.elapsed_time(ev1)) / e2e_steps
+        e2e_step_ms = [evk[k].elapsed_time(evk[k + 1]) for k in range(e2e_steps)]
+        # phase breakdown of one more e2e step (events on the stream; untimed)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
+        evs[0].record(stream)
+        if rank == 0:
+            alpha.copy_(values_h, non_blocking=True)
+        evs[1].record(stream)
+        if rank == 0:
+            g.hierarchize_(alpha)
+        x_d.copy_(x_h, non_blocking=True)
+        evs[2].record(stream)
+        if weak:
+            g.evaluate(alpha, x_d, out=y_d, workspace=ws)
+        else:
+            multi.evaluate_distributed(g, alpha, x_d, out=y_d, broadcast=world > 1)
+        evs[3].record(stream)
+        y_h.copy_(y_d, non_blocking=True)
+        evs[4].record(stream)
+        stream.synchronize()
+        e2e_phases = {"h2d_surplus_values": evs[0].elapsed_time(evs[1]),
+                      "hierarchize_and_h2d_queries": evs[1].elapsed_time(evs[2]),
+                      "order_and_evaluate": evs[2].elapsed_time(evs[3]), "d2h_results": evs[3].elapsed_time(evs[4])}
         own = perm[first:first + count].long().cpu()
         assert torch.equal(y_h[own], y.cpu()[own]), "e2e results differ from the device path"
         e2e = {"value": total_queries / (e2e_ms / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": (N * 8 if rank == 0 else 0) + m_batch * d * 8, "d2h_bytes_per_step": m_batch * 8,
-               "ms_per_step": e2e_ms, "steps": e2e_steps,
+               "ms_per_step": e2e_ms, "steps": e2e_steps, "step_ms_rank0": e2e_step_ms,
+               "breakdown_ms_rank0": e2e_phases,
                "path": "Grid.hierarchize_ + multi.evaluate_distributed (sg_sfc_order + sg_evaluate_ordered) "
                        "between pinned-host copies" if not weak else "Grid.evaluate between pinned-host copies"}
 

@@ -471,16 +471,13 @@ struct Trie {
 // One launch evaluates the level groups J0..J1 (compile time) for every
 // query; launches of consecutive ranges accumulate into y (accumulate = 0 for
 // the first range).  b0 = index3(J0), the offset of group J0.
-template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, class KN>
-__global__ void __launch_bounds__(NT, MINB)
-    k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
-                int n, uint32_t b0, int accumulate, T* __restrict__ y) {
+// One query per thread (q = its position in the order perm), shared-memory column tid.
+template <typename T, int D, int NM, int NT, int J0, int J1, class KN>
+__device__ __forceinline__ void eval_query(const T* __restrict__ alpha, const T* __restrict__ x,
+                                           const uint32_t* __restrict__ perm, uint32_t m, int n, uint32_t b0,
+                                           int accumulate, T* __restrict__ y, T* sm, int tid, uint32_t q) {
   using TR = Trie<T, D, NM, NT, KN>;
   constexpr int I = TR::I;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  T* sm = reinterpret_cast<T*>(smem_raw);
-  const int tid = threadIdx.x;
-  const uint32_t q = blockIdx.x * NT + tid;
   const bool active = q < m;
   const uint32_t src = active ? (perm ? perm[q] : q) : 0u;
 
@@ -554,6 +551,15 @@ __global__ void __launch_bounds__(NT, MINB)
     if (accumulate) r += (double)y[src];
     y[src] = bad ? T(NAN) : (T)r;
   }
+}
+
+template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, class KN>
+__global__ void __launch_bounds__(NT, MINB)
+    k_eval_trie(const T* __restrict__ alpha, const T* __restrict__ x, const uint32_t* __restrict__ perm, uint32_t m,
+                int n, uint32_t b0, int accumulate, T* __restrict__ y) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  eval_query<T, D, NM, NT, J0, J1, KN>(alpha, x, perm, m, n, b0, accumulate, y, reinterpret_cast<T*>(smem_raw),
+                                       threadIdx.x, blockIdx.x * NT + threadIdx.x);
 }
 
 template <typename T, int D, int NM, int NT, int MINB, int J0, int J1, class KN = Knobs>

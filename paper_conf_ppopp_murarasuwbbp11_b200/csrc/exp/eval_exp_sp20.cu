@@ -1,5 +1,5 @@
 // SP20 / SP20B: support-enumeration evaluation (eval_sparse.cuh) at d = 20, n <= 6, two CTA shapes
-#include "../eval_sparse.cuh"
+#include "eval_sparse.cuh"
 
 namespace sg {
 sg_status exp_SP20(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,

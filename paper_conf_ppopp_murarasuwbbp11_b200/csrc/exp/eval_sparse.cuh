@@ -1,4 +1,5 @@
-// eval_sparse.cuh -- the evaluation hot path (rows a2-a6; Alg. 7) for high-dimensional,
+// eval_sparse.cuh -- EXPERIMENT (libsg_exp.so only; measured slower than the product's S0 trie, profiles/r02_v9.txt):
+// the evaluation hot path (rows a2-a6; Alg. 7) for high-dimensional,
 // low-level grids (cfg5: d = 20, n = 6), enumerating each level vector by its SUPPORT.
 //
 // At d = 20 and n = 6 every level vector has at most 5 non-zero entries among 20, so the bijection-order
@@ -22,8 +23,8 @@
 // the cell digit k_t(v) (v <= 5 bits) in its 5 low mantissa bits (reading G21: a relative perturbation below
 // 2^-47 per factor), so one 8-byte shared load gives a factor and its digit.
 #pragma once
-#include "common.cuh"
-#include "eval_common.cuh"
+#include "../common.cuh"
+#include "../eval_common.cuh"
 
 namespace sg {
 namespace sparse {

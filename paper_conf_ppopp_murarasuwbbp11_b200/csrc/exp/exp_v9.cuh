@@ -5,6 +5,7 @@
 #include <type_traits>
 
 #include "../eval_trie.cuh"
+#include "exp_pw.cuh"
 
 namespace sg {
 namespace v9 {
@@ -26,14 +27,23 @@ struct KLow9 : trie::Knobs {
   static constexpr bool IDBL = ID;
   static constexpr bool GO = G;
 };
-template <class KL06, class KL, class KH, int NTL, int MBL, int NTH, int MBH>
+template <class KL06, class KL, class KH, int NTL, int MBL, int NTH, int MBH, bool PW = false>
 sg_status run(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,
               cudaStream_t s) {
   sg_status st = SG_OK;
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, NTL, MBL, 0, 6, KL06>(L, a, x, p, m, y, s);
-#define SG_R(J)                                                                                     \
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, NTL, MBL, J, J, KL>(L, a, x, p, m, y, s); \
-  if (st == SG_OK) st = trie::launch_range<double, 10, 11, NTH, MBH, J, J, KH>(L, a, x, p, m, y, s);
+  if constexpr (PW) {
+    if (st == SG_OK) st = pw::launch_range<double, 10, 11, NTL, MBL, 0, 6, KL06>(L, a, x, p, m, y, s);
+  } else {
+    if (st == SG_OK) st = trie::launch_range<double, 10, 11, NTL, MBL, 0, 6, KL06>(L, a, x, p, m, y, s);
+  }
+#define SG_R(J)                                                                                          \
+  if constexpr (PW) {                                                                                    \
+    if (st == SG_OK) st = pw::launch_range<double, 10, 11, NTL, MBL, J, J, KL>(L, a, x, p, m, y, s);     \
+    if (st == SG_OK) st = pw::launch_range<double, 10, 11, NTH, MBH, J, J, KH>(L, a, x, p, m, y, s);     \
+  } else {                                                                                               \
+    if (st == SG_OK) st = trie::launch_range<double, 10, 11, NTL, MBL, J, J, KL>(L, a, x, p, m, y, s);   \
+    if (st == SG_OK) st = trie::launch_range<double, 10, 11, NTH, MBH, J, J, KH>(L, a, x, p, m, y, s);   \
+  }
   SG_R(7) SG_R(8) SG_R(9) SG_R(10)
 #undef SG_R
   return st;
@@ -41,12 +51,12 @@ sg_status run(const Layout& L, const double* a, const double* x, const uint32_t*
 }  // namespace v9
 }  // namespace sg
 
-#define SG_V9(name, HZ, ID, G, NTL, MBL, NTH, MBH)                                                              \
+#define SG_V9(name, HZ, ID, G, NTL, MBL, NTH, MBH, ...)                                                              \
   namespace sg {                                                                                              \
   sg_status name(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,   \
                  cudaStream_t s) {                                                                            \
     using namespace v9;                                                                                       \
     using KH = typename std::conditional<G, KHighGO<4>, KHighN<4>>::type;                                     \
-    return run<KLow9<6, false, HZ, ID, G>, KLow9<4, false, HZ, ID, G>, KH, NTL, MBL, NTH, MBH>(L, a, x, p, m, y, s); \
+    return run<KLow9<6, false, HZ, ID, G>, KLow9<4, false, HZ, ID, G>, KH, NTL, MBL, NTH, MBH, ##__VA_ARGS__>(L, a, x, p, m, y, s); \
   }                                                                                                           \
   }

@@ -35,8 +35,9 @@ timeout 300 ncu --set full --clock-control none --import-source on -k regex:k_hi
   python bench.py --steps 1 --warmup 0 --m 100000 --no-e2e --no-cpu > gpurun_out/${TAG}_ncu_hier.log 2>&1
 timeout 120 python scripts/ncu_summary.py /tmp/${TAG}_hier.ncu-rep > gpurun_out/${TAG}_hier_ncu.txt 2>&1
 timeout 600 python scripts/bench_configs.py --reps 5 > gpurun_out/${TAG}_configs.txt 2>&1
-for TOOL in memcheck racecheck initcheck; do
-  timeout 900 compute-sanitizer --tool $TOOL --print-limit 50 python scripts/sanitize_run.py > gpurun_out/${TAG}_sanitizer_$TOOL.txt 2>&1
-  echo "exit $?" >> gpurun_out/${TAG}_sanitizer_$TOOL.txt
-done
+# compute-sanitizer is closed on this pool (exit 86, r02v9); the sanitizer driver stays in scripts/sanitize_run.py
+# for TOOL in memcheck racecheck initcheck; do
+#   timeout 900 compute-sanitizer --tool $TOOL --print-limit 50 python scripts/sanitize_run.py > gpurun_out/${TAG}_sanitizer_$TOOL.txt 2>&1
+#   echo "exit $?" >> gpurun_out/${TAG}_sanitizer_$TOOL.txt
+# done
 ls -la gpurun_out

@@ -1,4 +1,4 @@
-"""Host model of the support enumeration of csrc/eval_sparse.cuh (cfg5 kernel), pinned to the oracle.
+"""Host model of the support enumeration of csrc/exp/eval_sparse.cuh (cfg5 kernel), pinned to the oracle.
 
 The kernel enumerates the level vectors of a group by their highest non-zero dimension u and its level v,
 with the subspace offset off(u, B, v) = C(B+u, u) - C(B-v+u, u) and dimension u's cell digits at bit J - B.
