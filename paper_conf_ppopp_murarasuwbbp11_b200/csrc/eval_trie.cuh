@@ -87,6 +87,9 @@ struct Knobs {
   // hat values of dimension I (the innermost trie dimension) by doubling along its level loop, like the
   // dimensions above it, instead of a shared-memory row per level (NM - 1 fewer rows: more L1)
   static constexpr bool IDBL = false;
+  // experiment builds only: a CTA barrier at every level step of dimension SYNC (< 0: none), keeping the
+  // warps of a CTA in step through the enumeration (the trie's control flow is identical in every warp)
+  static constexpr int SYNC = -1;
 };
 struct KnobsS0 : Knobs {
   static constexpr bool S0 = true;
@@ -442,6 +445,7 @@ struct Trie {
       }
       T u = c.xs[xrow(t) * NT];
       for (int lt = 0; lt <= B; ++lt) {
+        if constexpr (KN::SYNC == t) __syncthreads();
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
         node<J, t - 1>(c, B - lt, P | (kt << SG), prod * hat_u(u));
         u = dbl_u(u);
