@@ -418,7 +418,7 @@ struct Trie {
         return;
       }
     }
-    if constexpr (S0 && I == 4 && t > I && J >= 1 && NM >= 2) {
+    if constexpr (S0 && t > I && J >= 1 && NM >= 2) {
       if (B == 1) {
         budget1<J, t>(c, P, prod);
         return;

@@ -23,3 +23,12 @@ struct KHighS : KHighN<RL> {
     return run<KLowS<6, SY>, KLowS<4, SY>, KHighS<4, SY>, 256, 2, 128, 3>(L, a, x, p, m, y, s);               \
   }                                                                                                            \
   }
+// barrier only in the small-block (SYL) or only in the large-block (SYH) launches
+#define SG_SYNC2(name, SYL, SYH)                                                                               \
+  namespace sg {                                                                                               \
+  sg_status name(const Layout& L, const double* a, const double* x, const uint32_t* p, uint64_t m, double* y,    \
+                 cudaStream_t s) {                                                                             \
+    using namespace v9;                                                                                        \
+    return run<KLowS<6, SYL>, KLowS<4, SYL>, KHighS<4, SYH>, 256, 2, 128, 3>(L, a, x, p, m, y, s);            \
+  }                                                                                                            \
+  }
