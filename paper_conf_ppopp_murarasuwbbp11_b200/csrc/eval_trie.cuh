@@ -87,8 +87,9 @@ struct Knobs {
   // hat values of dimension I (the innermost trie dimension) by doubling along its level loop, like the
   // dimensions above it, instead of a shared-memory row per level (NM - 1 fewer rows: more L1)
   static constexpr bool IDBL = false;
-  // experiment builds only: a CTA barrier at every level step of dimension SYNC (< 0: none), keeping the
-  // warps of a CTA in step through the enumeration (the trie's control flow is identical in every warp)
+  // a CTA barrier at every level step of dimension SYNC (< 0: none), keeping the warps of a CTA in step
+  // through the enumeration so that they share L1 lines (the trie's control flow is identical in every warp
+  // and every thread of the CTA, active or not, runs it: the barrier is uniform)
   static constexpr int SYNC = -1;
 };
 struct KnobsS0 : Knobs {

@@ -9,7 +9,8 @@
 // warps/SM (profiles/r02_split.txt).  v9: the small-block launches run as 256-thread CTAs (2 per SM:
 // 8 warps of neighbouring queries share the SM's L1) with hat rows of dimensions 2..4 only up to level
 // RMAX (18 KB less shared memory per 128 queries, so more L1) and the level-0 hats of dimensions 2..4 in
-// registers: +4.2%, +2.5% and +1.2% (profiles/r02_v9.txt).  Split across files only so that nvcc
+// registers: +4.2%, +2.5% and +1.2%; a CTA barrier per level step of dimension 9 keeps the warps of a CTA
+// in step (+1.3%) (profiles/r02_v9.txt).  Split across files only so that nvcc
 // compiles them in parallel.
 #include "eval_trie.cuh"
 
@@ -22,6 +23,7 @@ struct KLow : trie::Knobs {
   static constexpr int RMAX = RL;
   static constexpr int INNER = 5;
   static constexpr bool H0 = true;  // level-0 hats of dimensions 2..4 in registers (+1.2%, profiles/r02_v9.txt)
+  static constexpr int SYNC = 9;    // CTA barrier per level step of dimension 9 (+1.3%, profiles/r02_v9.txt)
 };
 // large blocks: blocks over dimensions 0..3 of every dimension-4 node with budget > RL (exactly the
 // complement: the nodes of budget <= RL are the small-block launch's blocks)
@@ -29,6 +31,7 @@ template <int RL>
 struct KHigh : trie::Knobs {
   static constexpr int RMIN = RL + 1;
   static constexpr bool RMIN_NODES_ONLY = true;
+  static constexpr int SYNC = 9;
 };
 }  // namespace d10
 

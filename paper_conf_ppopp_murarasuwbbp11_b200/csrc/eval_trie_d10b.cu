@@ -12,6 +12,7 @@ struct KLow : trie::Knobs {
   static constexpr int RMAX = RL;
   static constexpr int INNER = 5;
   static constexpr bool H0 = true;  // level-0 hats of dimensions 2..4 in registers (+1.2%, profiles/r02_v9.txt)
+  static constexpr int SYNC = 9;    // CTA barrier per level step of dimension 9 (+1.3%, profiles/r02_v9.txt)
 };
 // large blocks: blocks over dimensions 0..3 of every dimension-4 node with budget > RL (exactly the
 // complement: the nodes of budget <= RL are the small-block launch's blocks)
@@ -19,6 +20,7 @@ template <int RL>
 struct KHigh : trie::Knobs {
   static constexpr int RMIN = RL + 1;
   static constexpr bool RMIN_NODES_ONLY = true;
+  static constexpr int SYNC = 9;
 };
 }  // namespace d10b
 

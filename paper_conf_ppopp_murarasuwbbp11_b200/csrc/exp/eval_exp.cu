@@ -27,10 +27,8 @@ static sg_status d10_go(const Layout& L, const double* a, const double* x, const
   return st;
 }
 
-sg_status exp_SY8(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_SY9(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
-sg_status exp_SY8S(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
-sg_status exp_SY8H(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
+sg_status exp_BSY9(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_GOT(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 
 sg_status exp_SP20(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
@@ -52,10 +50,8 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   const double* xx = (const double*)x;
   double* yy = (double*)y;
   if (!strcmp(v, "GO4")) { *st = d10_go<4>(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SY8")) { *st = exp_SY8(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SY9")) { *st = exp_SY9(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SY8S")) { *st = exp_SY8S(L, a, xx, perm, m, yy, s); return true; }
-  if (!strcmp(v, "SY8H")) { *st = exp_SY8H(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "BSY9")) { *st = exp_BSY9(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GOT")) { *st = exp_GOT(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
