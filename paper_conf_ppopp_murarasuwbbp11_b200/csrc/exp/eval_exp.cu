@@ -31,6 +31,8 @@ sg_status exp_SY9(const Layout&, const double*, const double*, const uint32_t*, 
 sg_status exp_BSY9(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_LSY1(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_LSY2(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
+sg_status exp_LH4(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
+sg_status exp_LH42(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_GOT(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 
 sg_status exp_SP20(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
@@ -56,6 +58,8 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "BSY9")) { *st = exp_BSY9(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LSY1")) { *st = exp_LSY1(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LSY2")) { *st = exp_LSY2(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "LH4")) { *st = exp_LH4(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "LH42")) { *st = exp_LH42(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GOT")) { *st = exp_GOT(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
