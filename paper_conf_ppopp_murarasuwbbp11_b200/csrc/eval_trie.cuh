@@ -33,8 +33,9 @@
 // u = 2^l x - k_t(l), exact (reading G7).  The hat values of dimensions 0, 1
 // live in registers, those of dimensions 2, 3 and I in shared memory
 // ([row][lane], conflict-free, read once per block / slab / node);
-// dimensions > I recompute them along their loop (u <- frac(2u), exact for
-// x in [0,1), and still 0 outside).
+// dimensions > I recompute them along their loop (u <- frac(2u) and the hat
+// 2u or 2 - 2u, exact for x in [0,1]; a query with a coordinate outside the
+// cube is 0, reading G8).
 #pragma once
 #include "common.cuh"
 #include "eval_common.cuh"
@@ -298,15 +299,15 @@ struct Trie {
   // (23.7% no_instruction stalls at 70 terms, profiles/r01_v3_variants.txt):
   // only budget-0 sub-tries of dimensions > I are straight-line.
 
-  // hat value from u = 2^l x - k(l) (reading G7): max(0, 2 min(u, 1-u))
+  // hat value from u = 2^l x - k(l) in [0, 1] (reading G7): 2 min(u, 1-u) = 2u if 2u < 1, else 2 - 2u -- exact
+  // (2u is exact, 2 - 2u by Sterbenz).  Queries with a coordinate outside [0, 1] never use these values: their
+  // result is set to 0 (f_s = 0 outside the domain, reading G8), so no clamp is needed here.
   static __device__ __forceinline__ T hat_u(T u) {
     if constexpr (GO) return T(1);
-    const T w = T(1) - u;
-    const T mn = u < w ? u : w;
-    const T h = mn + mn;
-    return h > T(0) ? h : T(0);
+    const T t = u + u;
+    return t < T(1) ? t : T(2) - t;
   }
-  // u_{l+1} = frac(2 u_l), exact for u in [0, 1); stays outside [0,1) otherwise
+  // u_{l+1} = frac(2 u_l), exact for u in [0, 1]; u = 1 (x = 1, the clamped last cell) stays 1 (hat 0)
   static __device__ __forceinline__ T dbl_u(T u) {
     u = u + u;
     return u >= T(1) ? u - T(1) : u;
@@ -495,13 +496,14 @@ __device__ __forceinline__ void eval_query(const T* __restrict__ alpha, const T*
   T p0 = T(1);  // S0: running product of the level-0 hat values
   // ---- a2: finest cells of every dimension; hat values of every level of
   // dimensions 0..I (registers for 0, 1; shared memory for 2, 3, I)
-  bool bad = false;
+  bool bad = false, outside = false;
   const T fine = (T)(1u << (NM - 1));
   T h01[2][TR::PHN];  // D01: hat values of dimensions 0, 1 before their pairwise products
 #pragma unroll
   for (int t = 0; t < D; ++t) {
     const T xt = active ? x[(size_t)src * D + t] : T(0.5);
     bad |= isnan(xt);
+    outside |= !(xt >= T(0) && xt <= T(1));
     T kf = floor(xt * fine);
     kf = kf > T(0) ? kf : T(0);
     kf = kf < fine - T(1) ? kf : fine - T(1);
@@ -554,7 +556,7 @@ __device__ __forceinline__ void eval_query(const T* __restrict__ alpha, const T*
   if (active) {
     double r = c.res;
     if (accumulate) r += (double)y[src];
-    y[src] = bad ? T(NAN) : (T)r;
+    y[src] = bad ? T(NAN) : (outside ? T(0) : (T)r);
   }
 }
 

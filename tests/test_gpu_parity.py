@@ -354,11 +354,12 @@ def test_evaluate_edge_cases(P, torch, oracle, dt):
     check_eval(yg, yo, ao, TOL[dt], "grid points")
 
 
-@pytest.mark.parametrize("d,n", [(5, 8), (20, 6)])
+@pytest.mark.parametrize("d,n", [(5, 8), (20, 6), (10, 9)])
 def test_evaluate_edge_cases_specialised(P, torch, oracle, d, n):
     """Edge cases through the specialised trie kernels (cfg2 d=5 n=8; cfg5 d=20
     n=6 with the level-0 suffix products and the budget-1 Horner pass, whose
-    level-1 digit is taken from x >= 0.5): dyadic coordinates (cell
+    level-1 digit is taken from x >= 0.5; the cfg3 kernels at d=10 n=9, whose
+    trie dimensions take their hats by doubling): dyadic coordinates (cell
     boundaries at every level), 0.5 exactly, 1 - 2^-40, tiny, and rows with
     one coordinate on / outside the boundary (value 0) or NaN."""
     g = P.Grid(d, n)
@@ -374,11 +375,14 @@ def test_evaluate_edge_cases_specialised(P, torch, oracle, d, n):
     for r, v in bad.items():
         x[r, rng.integers(d)] = v
     x[6, d - 1] = np.nan
+    last = {7: 1.0, 8: -0.25, 9: 1.5, 10: 0.0}  # the last dimension (a trie dimension: hats by doubling)
+    for r, v in last.items():
+        x[r, d - 1] = v
     xt = torch.tensor(x, dtype=torch.float64, device="cuda")
     y = g.evaluate(alpha, xt).cpu().numpy()
     yo, ao = oracle.evaluate(d, n, alpha.cpu().numpy(), x)
     assert np.isnan(y[6]) and np.isnan(yo[6])
-    assert np.all(y[list(bad)] == 0.0)
+    assert np.all(y[list(bad) + list(last)] == 0.0)
     ok = ~np.isnan(yo)
     check_eval(y[ok], yo[ok], ao[ok], TOL["f64"], f"edge d={d}")
 
