@@ -15,7 +15,8 @@
 //     run-time amounts (sigma = j - R).
 // Cells k_t(l) = K_t >> (NMX-1-l), K_t = clamp(floor(2^{NMX-1} x_t)) (exact for l <= NMX-1);
 // hat values 2 min(u, 1-u) (reading G7); dimensions 0, 1 in registers, 2, 3 and I in shared memory,
-// dimensions > I by exact doubling along their loops -- as in eval_trie.cuh.
+// dimensions > I by exact doubling along their loops (2u or 2 - 2u, out-of-cube queries flagged and written
+// as 0), a CTA barrier per step of the top loop -- as in eval_trie.cuh.
 #pragma once
 #include "common.cuh"
 #include "eval_common.cuh"
@@ -128,11 +129,10 @@ struct GTrie {
   }
 #undef SG_GEN_CASE
 
+  // 2 min(u, 1-u) for u in [0, 1] as 2u or 2 - 2u (exact; queries outside the cube are written as 0, reading G8)
   static __device__ __forceinline__ T hat_u(T u) {
-    const T w = T(1) - u;
-    const T mn = u < w ? u : w;
-    const T h = mn + mn;
-    return h > T(0) ? h : T(0);
+    const T t = u + u;
+    return t < T(1) ? t : T(2) - t;
   }
   static __device__ __forceinline__ T dbl_u(T u) {
     u = u + u;
@@ -174,6 +174,9 @@ struct GTrie {
         for (int k = 0; k < lt0; ++k) u = dbl_u(u);
       }
       for (int lt = lt0; lt <= lt1; ++lt) {
+        // the top loop: a CTA barrier per level step keeps the CTA's warps in step through the enumeration
+        // (they share L1 lines; eval_trie.cuh Knobs::SYNC); uniform: every thread runs the same trie
+        if constexpr (t == D - 1 && NT > 32) __syncthreads();
         const uint32_t kt = c.K[t] >> (NM - 1 - lt);
         node<t - 1>(c, B - lt, P | (kt << SG), prod * hat_u(u));
         u = dbl_u(u);
@@ -198,12 +201,13 @@ __global__ void __launch_bounds__(NT, MINB)
   c.alpha = alpha;
   c.phs = sm + tid;
   c.xs = sm + (TR::SM_IN + TR::SM_PH) * NT + tid;
-  bool bad = false;
+  bool bad = false, outside = false;
   const T fine = (T)(1u << (NM - 1));
 #pragma unroll
   for (int t = 0; t < D; ++t) {
     const T xt = active ? x[(size_t)src * D + t] : T(0.5);
     bad |= isnan(xt);
+    outside |= !(xt >= T(0) && xt <= T(1));
     T kf = floor(xt * fine);
     kf = kf > T(0) ? kf : T(0);
     kf = kf < fine - T(1) ? kf : fine - T(1);
@@ -235,7 +239,7 @@ __global__ void __launch_bounds__(NT, MINB)
   if (active) {
     double r = c.res;
     if (accumulate) r += (double)y[src];
-    y[src] = bad ? T(NAN) : (T)r;
+    y[src] = bad ? T(NAN) : (outside ? T(0) : (T)r);
   }
 }
 

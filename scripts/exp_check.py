@@ -23,7 +23,9 @@ import sginputs as S  # noqa: E402
 import paper_conf_ppopp_murarasuwbbp11_b200 as P  # noqa: E402
 
 CFG = {"cfg2": (5, 8, 1_000_000), "cfg2p": (5, 10, 1_000_000), "cfg3": (10, 11, 10_000_000),
-       "cfg5": (20, 6, 1_000_000), "d16n5": (16, 5, 1_000_000), "d14n6": (14, 6, 1_000_000)}
+       "cfg5": (20, 6, 1_000_000), "d16n5": (16, 5, 1_000_000), "d14n6": (14, 6, 1_000_000),
+       "d11n10": (11, 10, 2_000_000), "d12n9": (12, 9, 2_000_000), "d8n11": (8, 11, 2_000_000),
+       "d6n12": (6, 12, 2_000_000)}
 
 
 def main():
