@@ -28,6 +28,7 @@ static sg_status d10_go(const Layout& L, const double* a, const double* x, const
 }
 
 sg_status exp_SY9(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
+sg_status exp_LIDBL(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_GOT(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 
 sg_status exp_SP20(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
@@ -65,6 +66,7 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   double* yy = (double*)y;
   if (!strcmp(v, "GO4")) { *st = d10_go<4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SY9")) { *st = exp_SY9(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "LIDBL")) { *st = exp_LIDBL(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GOT")) { *st = exp_GOT(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
