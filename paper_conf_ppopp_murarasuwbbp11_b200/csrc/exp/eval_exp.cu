@@ -29,12 +29,10 @@ static sg_status d10_go(const Layout& L, const double* a, const double* x, const
 
 sg_status exp_SY9(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_LIDBL(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
+sg_status exp_SIDBL(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_GOT(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 
 sg_status exp_SP20(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
-sg_status exp_D3T256(const Layout&, const float*, const float*, const uint32_t*, uint64_t, float*, cudaStream_t);
-sg_status exp_D3T512(const Layout&, const float*, const float*, const uint32_t*, uint64_t, float*, cudaStream_t);
-sg_status exp_D5T384(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_SP20B(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 // returns true if an experiment variant handled the call (the variants measured in r01/r02 before v9 are
 // recorded in profiles/r02_split.txt and profiles/r02_cfg5_variants.txt; their code is in the git history)
@@ -42,18 +40,7 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
                   sg_dtype dt, cudaStream_t s, sg_status* st) {
   const char* v = getenv("SG_EXP_VAR");
   if (!v) return false;
-  if (dt == SG_F32) {
-    if (L.d != 3 || L.n > 14) return false;
-    const float* af = (const float*)alpha;
-    if (!strcmp(v, "D3T256")) { *st = exp_D3T256(L, af, (const float*)x, perm, m, (float*)y, s); return true; }
-    if (!strcmp(v, "D3T512")) { *st = exp_D3T512(L, af, (const float*)x, perm, m, (float*)y, s); return true; }
-    return false;
-  }
   if (dt != SG_F64) return false;
-  if (L.d == 5 && L.n <= 10 && L.n > 8 && !strcmp(v, "D5T384")) {
-    *st = exp_D5T384(L, (const double*)alpha, (const double*)x, perm, m, (double*)y, s);
-    return true;
-  }
   if (L.d == 20 && L.n <= 6) {
     const double* a = (const double*)alpha;
     if (!strcmp(v, "SP20")) { *st = exp_SP20(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
@@ -67,6 +54,7 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (!strcmp(v, "GO4")) { *st = d10_go<4>(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "SY9")) { *st = exp_SY9(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "LIDBL")) { *st = exp_LIDBL(L, a, xx, perm, m, yy, s); return true; }
+  if (!strcmp(v, "SIDBL")) { *st = exp_SIDBL(L, a, xx, perm, m, yy, s); return true; }
   if (!strcmp(v, "GOT")) { *st = exp_GOT(L, a, xx, perm, m, yy, s); return true; }
   return false;
 }
