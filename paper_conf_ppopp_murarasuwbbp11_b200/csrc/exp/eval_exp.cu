@@ -33,6 +33,7 @@ sg_status exp_SIDBL(const Layout&, const double*, const double*, const uint32_t*
 sg_status exp_GOT(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 
 sg_status exp_SP20(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
+sg_status exp_D20ID(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 sg_status exp_SP20B(const Layout&, const double*, const double*, const uint32_t*, uint64_t, double*, cudaStream_t);
 // returns true if an experiment variant handled the call (the variants measured in r01/r02 before v9 are
 // recorded in profiles/r02_split.txt and profiles/r02_cfg5_variants.txt; their code is in the git history)
@@ -44,6 +45,7 @@ bool exp_dispatch(const Layout& L, const void* alpha, const void* x, const uint3
   if (L.d == 20 && L.n <= 6) {
     const double* a = (const double*)alpha;
     if (!strcmp(v, "SP20")) { *st = exp_SP20(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
+    if (!strcmp(v, "D20ID")) { *st = exp_D20ID(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
     if (!strcmp(v, "SP20B")) { *st = exp_SP20B(L, a, (const double*)x, perm, m, (double*)y, s); return true; }
     return false;
   }
